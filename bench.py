@@ -1,0 +1,429 @@
+"""Benchmark of the FDTD room-acoustics step (volume + FD-MM boundary + source/receivers).
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--impl rafd|reference] [--config C4]
+
+A "step" is one leapfrog time step of the whole hot path (SURVEY §8(a) rows
+a2-a6; the once-per-room classification a1 is timed inside `e2e`).  Workload at
+N=1: BASELINE.json configs[3], the C4 hall 1536x1024x704 (1.107e9 voxels), box,
+FD-MM with 3 branches and 8 materials, fp32.  N>1 (torchrun, one rank per GPU):
+weak scaling, the hall grows to 704*N planes, z-slab partitioned
+(rafd_slab_plan), one-plane NCCL halo exchange per step.  Inputs are synthetic
+and seeded (paper_conf_ipps_stoltzfushsld21_b200/inputs.py) and larger than L2.
+
+Prints ONE JSON line on rank 0.  `value` = inside-voxel updates of all ranks /
+max-over-ranks device time (CUDA events on the room's stream).
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import math
+import os
+import subprocess
+import sys
+import threading
+import time
+
+import numpy as np
+import torch
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+from paper_conf_ipps_stoltzfushsld21_b200 import inputs as I  # noqa: E402
+
+METRIC = "Gvoxel-updates/s (fp32/fp64) and % of HBM roofline at 1/2/4/8 B200"
+UNIT = "Gvox/s"
+LAM = 1.0 / math.sqrt(3.0)
+
+
+def peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        d = json.load(open(p))
+        return float(d["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs)"
+    return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
+
+
+class ClockSampler:
+    """nvidia-smi style sampling of SM clocks and throttle reasons via NVML."""
+
+    REASONS = {
+        "gpu_idle": 0x1, "applications_clocks_setting": 0x2, "sw_power_cap": 0x4,
+        "hw_slowdown": 0x8, "sync_boost": 0x10, "sw_thermal_slowdown": 0x20,
+        "hw_thermal_slowdown": 0x40, "hw_power_brake_slowdown": 0x80,
+    }
+
+    def __init__(self, device_index):
+        self.samples = []
+        self.reasons = set()
+        self.stop = threading.Event()
+        self.ok = False
+        try:
+            import pynvml
+            pynvml.nvmlInit()
+            self.nv = pynvml
+            self.h = pynvml.nvmlDeviceGetHandleByIndex(device_index)
+            self.max_mhz = pynvml.nvmlDeviceGetMaxClockInfo(self.h, pynvml.NVML_CLOCK_SM)
+            self.ok = True
+        except Exception as e:  # pragma: no cover
+            self.err = repr(e)
+
+    def _run(self):
+        nv = self.nv
+        while not self.stop.is_set():
+            try:
+                self.samples.append(nv.nvmlDeviceGetClockInfo(self.h, nv.NVML_CLOCK_SM))
+                r = nv.nvmlDeviceGetCurrentClocksEventReasons(self.h)
+                for k, bit in self.REASONS.items():
+                    if r & bit and k != "gpu_idle":
+                        self.reasons.add(k)
+            except Exception:
+                pass
+            time.sleep(0.02)
+
+    def __enter__(self):
+        if self.ok:
+            self.t = threading.Thread(target=self._run, daemon=True)
+            self.t.start()
+        return self
+
+    def __exit__(self, *a):
+        if self.ok:
+            self.stop.set()
+            self.t.join()
+
+    def result(self):
+        if not self.ok or not self.samples:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": [], "note": "nvml unavailable"}
+        return {"sm_mhz": float(np.median(self.samples)), "sm_max_mhz": float(self.max_mhz),
+                "reasons": sorted(self.reasons), "samples": len(self.samples)}
+
+
+def workload(cfg_name, nranks):
+    cfg = dict(I.CONFIGS[cfg_name])
+    nx, ny, nz = cfg["dims"]
+    if nranks > 1 and cfg_name != "C5":
+        nz = nz * nranks          # weak scaling: one C4-sized slab per GPU
+    cfg["room"] = (nx, ny, nz)
+    return cfg
+
+
+def slab_inputs(cfg, z0, z1, device):
+    """Box mask + region material map for planes [z0-1, z1] (clipped), generated
+    on `device`; returns (mask, matmap, mask_z0)."""
+    nx, ny, nz = cfg["room"]
+    lo, hi = max(0, z0 - 1), min(nz, z1 + 1)
+    assert cfg["shape"] == "box", "bench.py generates box halls slab by slab"
+    mask = torch.ones((hi - lo, ny, nx), dtype=torch.uint8, device=device)
+    if cfg["rule"] == "region":
+        mm = I.region_map_box(nx, ny, nz, lo, hi, M=cfg["M"], device=device)
+    else:
+        mm = torch.zeros_like(mask)
+    return mask, mm, lo
+
+
+def slab_plan_box(nx, ny, nz, precision, MB, nranks):
+    """The cost-weighted split of rafd_slab_plan for a BOX room, from the closed
+    form of its per-plane counts (end planes: all boundary; other planes: the
+    rim) so the 8e9-voxel mask never has to exist on the host.  Matches
+    rafd_slab_plan on boxes (tests/test_bench_host.py)."""
+    if nranks == 1:
+        return [(0, nz)]
+    s = precision // 8
+    a, b = nx - 2, ny - 2
+    nb_end = nx * ny
+    nb_mid = nx * ny - a * b
+    c_end = nx * ny + 3 * s * nx * ny + (6 + 3 * s + 4 * s * MB) * nb_end
+    c_mid = nx * ny + 3 * s * nx * ny + (6 + 3 * s + 4 * s * MB) * nb_mid
+    cost = np.full(nz, float(c_mid))
+    cost[0] = cost[-1] = c_end
+    pre = np.concatenate([[0.0], np.cumsum(cost)])
+    cuts = [0]
+    for k in range(1, nranks):
+        t = pre[-1] * k / nranks
+        e = int(np.searchsorted(pre, t))
+        if e > 0 and abs(pre[e - 1] - t) <= abs(pre[e] - t):
+            e -= 1
+        cuts.append(max(cuts[-1] + 1, min(e, nz - (nranks - k))))
+    cuts.append(nz)
+    return list(zip(cuts[:-1], cuts[1:]))
+
+
+def run_rafd(args, rank, world, local_rank):
+    from paper_conf_ipps_stoltzfushsld21_b200 import build, rafd
+    if rank == 0:
+        build.build()
+    if world > 1:
+        torch.distributed.barrier()
+    dev = torch.device("cuda", local_rank)
+    torch.cuda.set_device(dev)
+    cfg = workload(args.config, world)
+    nx, ny, nz = cfg["room"]
+    prec = cfg["precision"] if args.precision is None else args.precision
+    beta0, D, E, F = I.config_materials(cfg)
+    plan = slab_plan_box(nx, ny, nz, prec, cfg["MB"], world)
+    z0, z1 = plan[rank]
+    nccl_id = None
+    if world > 1:
+        obj = [rafd.rafd_nccl_unique_id() if rank == 0 else None]
+        torch.distributed.broadcast_object_list(obj, src=0)
+        nccl_id = obj[0]
+    stream = torch.cuda.Stream(device=dev)
+    mask, mm, mz0 = slab_inputs(cfg, z0, z1, dev)
+    t_c = time.perf_counter()
+    room = rafd.Room(mask, LAM, prec, beta0, D, E, F, matmap=mm, device=local_rank,
+                     stream=stream.cuda_stream, rank=rank, nranks=world, nccl_id=nccl_id,
+                     z_begin=z0, z_end=z1, mask_z0=mz0, dims=(nx, ny, nz))
+    t_create = time.perf_counter() - t_c
+    del mask, mm
+    torch.cuda.empty_cache()
+    room.set_source(I.source_position((nx, ny, nz)), I.impulse())
+    room.set_receivers(I.receiver_positions((nx, ny, nz)))
+    info = room.get_info()
+
+    # warm-up (also builds the CUDA graphs)
+    room.step(args.warmup)
+    room.synchronize()
+    room.read_receivers()
+
+    clk = ClockSampler(local_rank)
+    room.set_profiling(True)
+    n0 = room.launch_count()
+    ev0 = torch.cuda.Event(enable_timing=True)
+    ev1 = torch.cuda.Event(enable_timing=True)
+    if world > 1:
+        torch.distributed.barrier()
+    torch.cuda.synchronize()
+    with clk:
+        with torch.cuda.stream(stream):
+            ev0.record(stream)
+            room.step(args.steps)
+            ev1.record(stream)
+        torch.cuda.synchronize()
+    if world > 1:
+        torch.distributed.barrier()
+    ms = ev0.elapsed_time(ev1)
+    launches = room.launch_count() - n0
+    kt = room.get_kernel_times()
+    room.set_profiling(False)
+    rec = room.read_receivers()
+
+    t = torch.tensor([ms, float(info["n_inside"]), float(info["bytes_per_step"]), float(launches),
+                      kt["volume_ms"], kt["boundary_ms"], kt["other_ms"]], dtype=torch.float64,
+                     device=dev)
+    if world > 1:
+        mx = t.clone()
+        torch.distributed.all_reduce(mx, op=torch.distributed.ReduceOp.MAX)
+        sm = t.clone()
+        torch.distributed.all_reduce(sm, op=torch.distributed.ReduceOp.SUM)
+    else:
+        mx = sm = t
+    ms_max = float(mx[0])
+    n_in_total = float(sm[1])
+    bytes_total = float(sm[2])
+    value = n_in_total * args.steps / (ms_max * 1e-3) / 1e9
+
+    out = None
+    if rank == 0:
+        peak, peak_src = peaks()
+        vol_ms = kt["volume_ms"] / max(1, kt["volume_launches"])
+        bnd_ms = kt["boundary_ms"] / max(1, kt["boundary_launches"])
+        vol_gbs = info["volume_bytes"] / (vol_ms * 1e-3) / 1e9
+        bnd_gbs = info["boundary_bytes"] / (bnd_ms * 1e-3) / 1e9 if info["n_boundary"] else None
+        step_gbs = bytes_total * args.steps / (ms_max * 1e-3) / 1e9 / world
+        traffic = None
+        tp = os.path.join(ROOT, "profiles", "volume_traffic.json")
+        if os.path.exists(tp):
+            try:
+                traffic = json.load(open(tp)).get("dram_bytes_per_launch")
+            except Exception:
+                traffic = None
+        out = {
+            "metric": METRIC, "value": round(value, 3), "unit": UNIT, "n_gpus": world,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(ms_max / args.steps, 4),
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
+            "dtype": "f32" if prec == 32 else "f64",
+            "data": "synthetic (seeded box hall, region materials, seeded FD tables, impulse source)",
+            "config": {
+                "workload": f"{args.config}: {nx}x{ny}x{nz} box hall, FD-MM MB={cfg['MB']} M={cfg['M']}, "
+                            f"fp{prec}" + (f", {world} z-slabs" if world > 1 else ""),
+                "room_dims_xyz": [nx, ny, nz], "n_inside": int(n_in_total),
+                "n_boundary_rank0": info["n_boundary"], "parallelism": f"z-slab x{world}",
+                "l2": "inputs larger than L2 (working set %.1f GB/GPU vs 126 MB L2)" % (info["device_bytes"] / 1e9),
+                "timed": "profiled launches (CUDA events around every kernel) on the room stream",
+            },
+            "roofline": {
+                "bound": "hbm", "kernel": "k_volume", "achieved": round(vol_gbs, 1), "peak": peak,
+                "unit": "GB/s", "frac": round(vol_gbs / peak, 4), "traffic": traffic,
+                "algorithmic_bytes_per_launch": info["volume_bytes"],
+                "avg_launch_ms": round(vol_ms, 5), "peak_source": peak_src,
+            },
+            "kernels": {
+                "volume_ms_per_step": round(vol_ms, 5), "boundary_ms_per_step": round(bnd_ms, 5),
+                "other_ms_per_step": round(kt["other_ms"] / max(1, kt["other_launches"]), 5),
+                "boundary_gbs": None if bnd_gbs is None else round(bnd_gbs, 1),
+                "boundary_share": round(bnd_ms / (ms_max / args.steps), 4),
+                "step_algorithmic_gbs_per_gpu": round(step_gbs, 1),
+                "step_frac_of_peak": round(step_gbs / peak, 4),
+            },
+            "gpu_launches": int(launches),
+            "clocks": clk.result(),
+            "create_s": round(t_create, 3),
+            "receivers_checksum": float(np.abs(rec).sum()),
+        }
+    room.destroy()
+    del room
+    torch.cuda.synchronize()
+    torch.cuda.empty_cache()
+    e2e = run_e2e(args, cfg, prec, beta0, D, E, F, rank, world, local_rank, plan, nccl_id is not None)
+    if rank == 0:
+        out["e2e"] = e2e
+    return out
+
+
+def run_e2e(args, cfg, prec, beta0, D, E, F, rank, world, local_rank, plan, multi):
+    """End to end through the public API with HOST buffers: create the room from
+    pinned host mask/matmap (H2D + on-device classification), set source and
+    receivers, then every step: rafd_step(1) and rafd_read_receivers (D2H of the
+    step's receiver samples); destroy.  Wall clock, max over ranks."""
+    from paper_conf_ipps_stoltzfushsld21_b200 import rafd
+    nx, ny, nz = cfg["room"]
+    z0, z1 = plan[rank]
+    mask_d, mm_d, mz0 = slab_inputs(cfg, z0, z1, torch.device("cuda", local_rank))
+    mask_h = torch.empty(mask_d.shape, dtype=torch.uint8, pin_memory=True)
+    mm_h = torch.empty(mm_d.shape, dtype=torch.uint8, pin_memory=True)
+    mask_h.copy_(mask_d)
+    mm_h.copy_(mm_d)
+    del mask_d, mm_d
+    torch.cuda.empty_cache()
+    nccl_id = None
+    if multi:
+        obj = [rafd.rafd_nccl_unique_id() if rank == 0 else None]
+        torch.distributed.broadcast_object_list(obj, src=0)
+        nccl_id = obj[0]
+    sig = I.impulse()
+    rcv = I.receiver_positions((nx, ny, nz))
+    steps = args.steps
+    if world > 1:
+        torch.distributed.barrier()
+    torch.cuda.synchronize()
+    t0 = time.perf_counter()
+    room = rafd.Room(mask_h.numpy(), LAM, prec, beta0, D, E, F, matmap=mm_h.numpy(), device=local_rank,
+                     rank=rank, nranks=world, nccl_id=nccl_id, z_begin=z0, z_end=z1, mask_z0=mz0,
+                     dims=(nx, ny, nz))
+    room.set_source(I.source_position((nx, ny, nz)), sig)
+    room.set_receivers(rcv)
+    d2h = 0
+    for _ in range(steps):
+        room.step(1)
+        r = room.read_receivers(cap=1)
+        d2h += r.shape[0] * r.shape[1] * (prec // 8)
+    room.synchronize()
+    t1 = time.perf_counter()
+    n_in = room.get_info()["n_inside"]
+    room.destroy()
+    el = torch.tensor([t1 - t0, float(n_in)], dtype=torch.float64, device=torch.device("cuda", local_rank))
+    if world > 1:
+        mx = el.clone()
+        torch.distributed.all_reduce(mx, op=torch.distributed.ReduceOp.MAX)
+        sm = el.clone()
+        torch.distributed.all_reduce(sm, op=torch.distributed.ReduceOp.SUM)
+        tmax, n_tot = float(mx[0]), float(sm[1])
+    else:
+        tmax, n_tot = float(el[0]), float(el[1])
+    h2d = mask_h.numel() + mm_h.numel() + sig.size * 8
+    return {"value": round(n_tot * steps / tmax / 1e9, 3), "unit": UNIT,
+            "h2d_bytes_per_step": int(h2d // steps), "d2h_bytes_per_step": int(d2h // steps),
+            "wall_s": round(tmax, 3),
+            "includes": "rafd_create from pinned host mask+matmap (H2D, device classification), "
+                        "set_source/set_receivers, per step rafd_step(1)+rafd_read_receivers (D2H), destroy"}
+
+
+def oracle_sample(cfg, nplanes):
+    """Bounded sample of the workload for the CPU oracle: the same x-y section,
+    `nplanes` planes (a box of nx x ny x nplanes), same materials."""
+    from oracle import orc
+    nx, ny, nz = cfg["room"]
+    mask = I.box_mask(nx, ny, nplanes)
+    mm = I.material_map(mask, cfg["rule"], cfg["M"]).numpy()
+    beta0, D, E, F = I.config_materials(cfg)
+    prec = cfg["precision"]
+    r = orc.OracleRoom(mask.numpy(), LAM, prec, beta0, D, E, F, matmap=mm)
+    r.set_source(I.source_position((nx, ny, nplanes)), I.impulse())
+    r.set_receivers(I.receiver_positions((nx, ny, nplanes)))
+    return r, (nx, ny, nplanes)
+
+
+def cpu_baseline(cfg, seconds=12.0, nplanes=16):
+    r, dims = oracle_sample(cfg, nplanes)
+    n_in = r.info()["n_inside"]
+    r.step(1)
+    t0 = time.perf_counter()
+    n = 0
+    while time.perf_counter() - t0 < seconds:
+        r.step(1)
+        n += 1
+    dt = time.perf_counter() - t0
+    return {"value": round(n_in * n / dt / 1e9, 5), "unit": UNIT, "cores": 1, "kind": "oracle",
+            "sample": f"{dims[0]}x{dims[1]}x{dims[2]} box crop of the workload (same materials), "
+                      f"{n} steps in {dt:.1f} s, single-threaded C oracle (-O2 -ffp-contract=off)"}
+
+
+def run_reference(args):
+    """--impl reference: the CPU oracle as it stands (the only reference this
+    tier has), each step a bounded sample of the workload."""
+    cfg = workload(args.config, 1)
+    nplanes = 16
+    r, dims = oracle_sample(cfg, nplanes)
+    n_in = r.info()["n_inside"]
+    r.step(args.warmup)
+    t0 = time.perf_counter()
+    r.step(args.steps)
+    dt = time.perf_counter() - t0
+    v = n_in * args.steps / dt / 1e9
+    sample = f"{dims[0]}x{dims[1]}x{dims[2]} box crop of {args.config} (same x-y section and materials)"
+    return {"impl": "reference", "metric": METRIC, "value": round(v, 5), "unit": UNIT, "n_gpus": 0,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(dt / args.steps * 1e3, 3),
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
+            "dtype": "f32" if cfg["precision"] == 32 else "f64", "data": "synthetic",
+            "config": {"workload": f"{args.config} sample: {sample}"},
+            "cpu_baseline": {"value": round(v, 5), "unit": UNIT, "cores": 1, "kind": "oracle",
+                             "sample": sample},
+            "e2e": {"value": round(v, 5), "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=200)
+    ap.add_argument("--warmup", type=int, default=5)
+    ap.add_argument("--impl", default="rafd", choices=["rafd", "reference"])
+    ap.add_argument("--config", default="C4")
+    ap.add_argument("--precision", type=int, default=None)
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    args = ap.parse_args()
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local_rank = int(os.environ.get("LOCAL_RANK", "0"))
+    if args.impl == "reference":
+        if rank == 0:
+            print(json.dumps(run_reference(args)), flush=True)
+        return
+    if world > 1:
+        torch.cuda.set_device(local_rank)
+        torch.distributed.init_process_group("nccl", device_id=torch.device("cuda", local_rank))
+    out = run_rafd(args, rank, world, local_rank)
+    if rank == 0:
+        if world == 1 and not args.no_cpu_baseline:
+            out["cpu_baseline"] = cpu_baseline(workload(args.config, 1))
+        else:
+            out["cpu_baseline"] = None
+        print(json.dumps(out), flush=True)
+    if world > 1:
+        torch.distributed.barrier()
+        torch.distributed.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

@@ -1,0 +1,110 @@
+// internal.cuh -- shared definitions of the CUDA library (not part of the ABI).
+#pragma once
+
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include <string>
+#include <vector>
+
+#include "../../include/rafd.h"
+
+namespace rafd {
+
+// ------------------------------------------------------------------ arithmetic
+// Correctly rounded single operations (no FMA contraction), DESIGN.md §4.
+template <typename T> struct rn;
+template <> struct rn<float> {
+    static __device__ __forceinline__ float add(float a, float b) { return __fadd_rn(a, b); }
+    static __device__ __forceinline__ float sub(float a, float b) { return __fsub_rn(a, b); }
+    static __device__ __forceinline__ float mul(float a, float b) { return __fmul_rn(a, b); }
+    static __device__ __forceinline__ float div(float a, float b) { return __fdiv_rn(a, b); }
+};
+template <> struct rn<double> {
+    static __device__ __forceinline__ double add(double a, double b) { return __dadd_rn(a, b); }
+    static __device__ __forceinline__ double sub(double a, double b) { return __dsub_rn(a, b); }
+    static __device__ __forceinline__ double mul(double a, double b) { return __dmul_rn(a, b); }
+    static __device__ __forceinline__ double div(double a, double b) { return __ddiv_rn(a, b); }
+};
+
+// ------------------------------------------------------------------ grid layout
+// Padded grid in HBM: (lnz+2) planes x (ny+2) rows x pitch
+// elements.  Room voxel (x, y, zl) (zl slab-local, 0..lnz-1) lives at
+//   (zl+1)*plane + (y+1)*pitch + xo + x
+// with xo = 16/sizeof(T) so every interior row starts 16-byte aligned; the x
+// halo cells are xo-1 and xo+nx; pitch is a multiple of 128 bytes.  The uint8
+// K grid uses the same element indexing.
+struct Grid {
+    int32_t nx, ny, lnz;
+    int32_t xo;
+    int64_t pitch, plane, total;
+};
+
+// Device control block for the per-step source / receivers (read by the
+// src/rcv kernel so that CUDA graphs never need re-capturing).
+template <typename T> struct Ctl {
+    int64_t n;          // step counter (index into sig)
+    int64_t rec_count;  // samples recorded since the last read
+    int64_t rec_cap;    // capacity of rec (rows)
+    T *rec;             // [rec_cap][nrcv]
+    const T *sig;       // [sig_len]
+    int64_t sig_len;
+    int64_t src_pos;    // padded index or -1
+    int32_t nrcv;
+    int32_t pad_;
+    const int64_t *rcv_pos;  // [nrcv] padded indices
+};
+
+struct KernelTimes {
+    double volume_ms = 0, boundary_ms = 0, other_ms = 0;
+    int64_t volume_n = 0, boundary_n = 0, other_n = 0;
+};
+
+// ------------------------------------------------------------------ launchers
+// (each returns cudaGetLastError() of its launch)
+template <typename T>
+cudaError_t launch_volume(const Grid &g, const T *cur, T *nxt, const uint8_t *K, double lambda,
+                          int z_lo, int z_hi, cudaStream_t s);
+template <typename T>
+cudaError_t launch_boundary(int MB, bool idx64, const void *bpos, const uint8_t *Kb,
+                            const uint8_t *matb, int64_t i_lo, int64_t i_hi, int64_t Nb, T *unext,
+                            const T *ucur, T *ub_prev, T *g, T *v, const T *tab, int M,
+                            double lambda, cudaStream_t s);
+template <typename T>
+cudaError_t launch_src_rcv(T *unext, Ctl<T> *ctl, cudaStream_t s);
+
+// classification: flags -> K (in place, bit 7 trick), counts, compaction
+cudaError_t launch_scatter_mask(const Grid &g, const uint8_t *mask_chunk, int zp0, int nzc,
+                                uint8_t *K, cudaStream_t s);
+cudaError_t launch_count_k(const Grid &g, uint8_t *K, cudaStream_t s);
+cudaError_t launch_finish_k(const Grid &g, uint8_t *K, unsigned long long *hist8,
+                            cudaStream_t s);
+cudaError_t launch_row_counts64(const Grid &g, const uint8_t *K, int64_t *counts, cudaStream_t s);
+cudaError_t launch_compact(const Grid &g, const uint8_t *K, const int64_t *row_off, int64_t zglob0,
+                           int32_t ny_glob, int32_t nx_glob, bool idx64, void *bpos,
+                           int64_t *bidx, uint8_t *Kb, cudaStream_t s);
+cudaError_t launch_gather_mat(const uint8_t *matmap_chunk, int64_t canon0, const int64_t *bidx,
+                              int64_t i_lo, int64_t i_hi, uint8_t *matb, int M,
+                              unsigned int *bad_flag, cudaStream_t s);
+cudaError_t exclusive_scan_rows64(const int64_t *counts, int64_t *row_off, int64_t n, void *tmp,
+                                  size_t *tmp_bytes, cudaStream_t s);
+
+// fields in / out (canonical <-> padded), chunked over planes
+template <typename T>
+cudaError_t launch_field_in(const Grid &g, const T *src_chunk, int z0, int nzc, const uint8_t *K,
+                            T *dst, cudaStream_t s);
+template <typename T>
+cudaError_t launch_field_out(const Grid &g, const T *src, int z0, int nzc, T *dst_chunk,
+                             cudaStream_t s);
+template <typename T>
+cudaError_t launch_gather_ub(const void *bpos, bool idx64, int64_t Nb, const T *u, T *ub,
+                             cudaStream_t s);
+template <typename T>
+cudaError_t launch_energy(const Grid &g, const T *un1, const T *un, const uint8_t *K, double *acc,
+                          cudaStream_t s);
+template <typename T>
+cudaError_t launch_energy_bnd(const uint8_t *Kb, const uint8_t *matb, int64_t Nb, int MB,
+                              const T *v, const T *gst, const double *DF, int M, double lambda,
+                              double *acc, cudaStream_t s);
+
+}  // namespace rafd

@@ -1,0 +1,990 @@
+// room.cu -- the C-ABI (include/rafd.h): room lifetime, classification
+// orchestration, the per-step launch sequence (row a6: time-level rotation),
+// CUDA-graph replay, profiling, and the host-side slab planner.
+//
+// Per step (Listing 5: volume kernel, then the boundary
+// kernel updating the volume in place, "executed iteratively"):
+//   k_volume   (u[cur] -> u[cur^1], in place over u^{n-1})
+//   k_boundary (nodes of the slab; FI-MM or FD-MM; refreshes ub_prev)
+//   k_src_rcv  (soft source + receivers, reading R10)
+//   [slab halo exchange over NCCL, multi-GPU only]
+//   cur ^= 1
+#include <dlfcn.h>
+#include <math.h>
+#include <stdarg.h>
+#include <stdio.h>
+#include <string.h>
+
+#include <algorithm>
+#include <cfloat>
+#include <string>
+#include <vector>
+
+#include "internal.cuh"
+#include "halo.h"
+
+using namespace rafd;
+
+// ------------------------------------------------------------------ errors
+static thread_local std::string g_err;
+
+static int set_err(int code, const char *fmt, ...)
+{
+    char buf[512];
+    va_list ap;
+    va_start(ap, fmt);
+    vsnprintf(buf, sizeof buf, fmt, ap);
+    va_end(ap);
+    g_err = buf;
+    return code;
+}
+
+#define CK(call)                                                                        \
+    do {                                                                                \
+        cudaError_t e_ = (call);                                                        \
+        if (e_ != cudaSuccess)                                                          \
+            return set_err(e_ == cudaErrorMemoryAllocation ? RAFD_E_NOMEM : RAFD_E_CUDA, \
+                           "%s: %s (%s:%d)", #call, cudaGetErrorString(e_), __FILE__,   \
+                           __LINE__);                                                   \
+    } while (0)
+
+static bool is_device_ptr(const void *p)
+{
+    if (!p) return false;
+    cudaPointerAttributes a;
+    if (cudaPointerGetAttributes(&a, p) != cudaSuccess) {
+        cudaGetLastError();
+        return false;
+    }
+    return a.type == cudaMemoryTypeDevice || a.type == cudaMemoryTypeManaged;
+}
+
+// ------------------------------------------------------------------ the room
+struct rafd_room {
+    int device = 0;
+    cudaStream_t stream = nullptr, cap_stream = nullptr;
+    bool own_stream = false;
+    int prec = 32, M = 1, MB = 0;
+    size_t s = 4;
+    int32_t nx = 0, ny = 0, nz = 0;  // room
+    int32_t z0 = 0, z1 = 0;          // owned planes
+    int rank = 0, nranks = 1;
+    double lambda = 0;
+    Grid g{};
+    int nsm = 148;
+    void *u[2] = {nullptr, nullptr};
+    int cur = 0;  // u[cur] = u^n
+    uint8_t *K = nullptr;
+    int64_t nb = 0;
+    bool idx64 = false;
+    void *bpos = nullptr;
+    int64_t *bidx = nullptr;
+    uint8_t *Kb = nullptr, *matb = nullptr;
+    void *ub = nullptr, *gst = nullptr, *vst = nullptr;
+    void *tab = nullptr;   // T: beta[M] | BI | D | DI | F  ([M*MB] each)
+    double *DF = nullptr;  // double D | F for the energy hook
+    void *ctl = nullptr;   // Ctl<T>
+    void *sig = nullptr;
+    int64_t *rcv_pos = nullptr;
+    void *rec = nullptr;
+    int64_t rec_cap = 0, rec_count = 0;
+    int32_t nrcv = 0;
+    int64_t steps = 0;
+    int64_t k_hist[7] = {0};
+    int64_t isolated = 0, n_inside = 0;
+    int64_t device_bytes = 0;
+    int64_t launches = 0;
+    // CUDA graphs of G steps, one per starting parity
+    static const int G = 16;
+    cudaGraphExec_t graph[2] = {nullptr, nullptr};
+    int graph_kernels = 0;
+    // profiling
+    bool profiling = false;
+    struct Ev {
+        int kind;
+        cudaEvent_t a, b;
+    };
+    std::vector<Ev> evs;
+    std::vector<cudaEvent_t> ev_pool;
+    KernelTimes kt;
+    // multi-GPU halo exchange
+    Halo *halo = nullptr;
+};
+
+template <typename T> static Ctl<T> *ctl_of(rafd_room *r) { return (Ctl<T> *)r->ctl; }
+
+static int dmalloc(rafd_room *r, void **p, size_t bytes)
+{
+    if (bytes == 0) bytes = 16;
+    cudaError_t e = cudaMalloc(p, bytes);
+    if (e != cudaSuccess) {
+        cudaGetLastError();
+        *p = nullptr;
+        return set_err(RAFD_E_NOMEM, "cudaMalloc(%zu bytes): %s", bytes, cudaGetErrorString(e));
+    }
+    r->device_bytes += (int64_t)bytes;
+    return RAFD_OK;
+}
+
+// ------------------------------------------------------------------ validation
+static int validate(const rafd_room_desc *d)
+{
+    if (!d) return set_err(RAFD_E_INVAL, "null descriptor");
+    if (!d->mask) return set_err(RAFD_E_INVAL, "null mask");
+    if (d->nx < 1 || d->ny < 1 || d->nz < 1) return set_err(RAFD_E_INVAL, "dims must be >= 1");
+    if (d->precision != 32 && d->precision != 64) return set_err(RAFD_E_INVAL, "precision must be 32 or 64");
+    if (!d->mat) return set_err(RAFD_E_INVAL, "null materials");
+    const rafd_materials *m = d->mat;
+    if (m->n_materials < 1 || m->n_materials > RAFD_MAX_MATERIALS) return set_err(RAFD_E_INVAL, "n_materials must be in 1..256");
+    if (m->n_branches < 0 || m->n_branches > RAFD_MAX_BRANCHES) return set_err(RAFD_E_INVAL, "n_branches must be in 0..8");
+    if (!m->beta0) return set_err(RAFD_E_INVAL, "beta0 is required");
+    if (m->n_branches > 0 && (!m->D || !m->E || !m->F)) return set_err(RAFD_E_INVAL, "D, E, F are required when n_branches > 0");
+    // reading R1
+    if (!(d->lambda > 0.0) || !std::isfinite(d->lambda)) return set_err(RAFD_E_UNSTABLE, "lambda must be finite and > 0");
+    if (d->lambda * d->lambda > (1.0 / 3.0) * (1.0 + 4.0 * DBL_EPSILON)) return set_err(RAFD_E_UNSTABLE, "lambda^2 > 1/3");
+    // reading R5: passivity
+    const int M = m->n_materials, MB = m->n_branches;
+    for (int i = 0; i < M; i++) {
+        if (!(m->beta0[i] >= 0.0) || !std::isfinite(m->beta0[i])) return set_err(RAFD_E_NONPASSIVE, "beta0[%d] must be finite and >= 0", i);
+        for (int b = 0; b < MB; b++) {
+            const double D = m->D[i * MB + b], E = m->E[i * MB + b], F = m->F[i * MB + b];
+            if (!(D >= 0.0 && E >= 0.0 && F >= 0.0) || !std::isfinite(D) || !std::isfinite(E) || !std::isfinite(F))
+                return set_err(RAFD_E_NONPASSIVE, "D, E, F of material %d branch %d must be finite and >= 0", i, b);
+        }
+    }
+    if (d->mask_z0 < 0 || d->mask_z0 > std::max(0, (d->nranks > 1 ? d->z_begin : 0) - 1))
+        return set_err(RAFD_E_INVAL, "mask_z0 must be <= the first plane read (z_begin-1, clipped)");
+    if (d->nranks > 1) {
+        if (d->rank < 0 || d->rank >= d->nranks) return set_err(RAFD_E_INVAL, "rank out of range");
+        if (!(d->z_begin >= 0 && d->z_begin < d->z_end && d->z_end <= d->nz))
+            return set_err(RAFD_E_INVAL, "slab [z_begin, z_end) must be a non-empty range of planes (use rafd_slab_plan)");
+    }
+    return RAFD_OK;
+}
+
+// Derived per-material coefficients (reading R5), in double, then rounded to T.
+template <typename T>
+static void build_tables(const rafd_materials *m, std::vector<T> &tab, std::vector<double> &DF)
+{
+    const int M = m->n_materials, MB = m->n_branches;
+    tab.assign((size_t)M * (1 + 4 * MB), (T)0);
+    DF.assign((size_t)2 * M * MB + 1, 0.0);
+    T *beta = tab.data(), *BI = beta + M, *D = BI + M * MB, *DI = D + M * MB, *F = DI + M * MB;
+    for (int i = 0; i < M; i++) {
+        double bsum = m->beta0[i];
+        for (int b = 0; b < MB; b++) {
+            const int k = i * MB + b;
+            const double d = m->D[k], e = m->E[k], f = m->F[k];
+            const bool unused = (d == 0.0 && e == 0.0 && f == 0.0);
+            const double bi = unused ? 0.0 : 1.0 / ((2.0 * d + e) + f);
+            const double di = (2.0 * d - e) - f;
+            bsum = bsum + bi;
+            BI[k] = (T)bi;
+            D[k] = (T)d;
+            DI[k] = (T)di;
+            F[k] = (T)f;
+            DF[k] = d;
+            DF[(size_t)M * MB + k] = f;
+        }
+        beta[i] = (T)bsum;
+    }
+}
+
+// Copy nplanes planes (each plane_bytes) starting at plane zg0 of a host or
+// device array into `staging` chunk by chunk and call fn(chunk_ptr, zg, n).
+// `src` holds planes [src_z0, ...) of the room.
+template <typename Fn>
+static int for_plane_chunks(rafd_room *r, const void *src, int src_z0, bool dev, size_t plane_bytes,
+                            int zg0, int nplanes, void *staging, size_t staging_bytes, Fn fn)
+{
+    if (nplanes <= 0) return RAFD_OK;
+    if (dev) return fn((const char *)src + (size_t)(zg0 - src_z0) * plane_bytes, zg0, nplanes);
+    int per = (int)std::max<size_t>(1, staging_bytes / plane_bytes);
+    for (int z = zg0; z < zg0 + nplanes; z += per) {
+        const int n = std::min(per, zg0 + nplanes - z);
+        CK(cudaMemcpyAsync(staging, (const char *)src + (size_t)(z - src_z0) * plane_bytes, (size_t)n * plane_bytes,
+                           cudaMemcpyHostToDevice, r->stream));
+        int rc = fn(staging, z, n);
+        if (rc) return rc;
+        CK(cudaStreamSynchronize(r->stream));  // staging reused by the next chunk
+    }
+    return RAFD_OK;
+}
+
+static const size_t kStagingBytes = 256ull << 20;
+
+template <typename T> static int create_t(rafd_room *r, const rafd_room_desc *d)
+{
+    const int64_t nxny = (int64_t)r->nx * r->ny;
+    Grid &g = r->g;
+    g.nx = r->nx;
+    g.ny = r->ny;
+    g.lnz = r->z1 - r->z0;
+    g.xo = (int)(16 / sizeof(T));
+    const int64_t align = 128 / (int64_t)sizeof(T);
+    g.pitch = ((g.xo + r->nx + 1 + align - 1) / align) * align;
+    g.plane = g.pitch * (r->ny + 2);
+    g.total = g.plane * (g.lnz + 2);
+    r->idx64 = g.total >= (int64_t)UINT32_MAX;
+
+    int rc;
+    if ((rc = dmalloc(r, (void **)&r->K, (size_t)g.total + 64))) return rc;
+    for (int k = 0; k < 2; k++)
+        if ((rc = dmalloc(r, &r->u[k], (size_t)g.total * sizeof(T) + 64))) return rc;
+    CK(cudaMemsetAsync(r->K, 0, (size_t)g.total + 64, r->stream));
+    for (int k = 0; k < 2; k++) CK(cudaMemsetAsync(r->u[k], 0, (size_t)g.total * sizeof(T) + 64, r->stream));
+
+    // ---- classification (row a1)
+    const bool mdev = is_device_ptr(d->mask);
+    void *staging = nullptr;
+    if ((!mdev || (d->matmap && !is_device_ptr(d->matmap))) &&
+        (rc = dmalloc(r, &staging, kStagingBytes)))
+        return rc;
+    const int zlo = std::max(0, r->z0 - 1), zhi = std::min(r->nz, r->z1 + 1);  // incl. ghost planes
+    const int mz0 = d->mask_z0;
+    rc = for_plane_chunks(r, d->mask, mz0, mdev, (size_t)nxny, zlo, zhi - zlo, staging, kStagingBytes,
+                          [&](const void *chunk, int zg, int n) -> int {
+                              CK(launch_scatter_mask(g, (const uint8_t *)chunk, zg - r->z0 + 1, n, r->K, r->stream));
+                              return RAFD_OK;
+                          });
+    if (rc) return rc;
+    CK(launch_count_k(g, r->K, r->stream));
+    unsigned long long *hist = nullptr;
+    if ((rc = dmalloc(r, (void **)&hist, 8 * sizeof(unsigned long long) + sizeof(unsigned)))) return rc;
+    CK(cudaMemsetAsync(hist, 0, 8 * sizeof(unsigned long long) + sizeof(unsigned), r->stream));
+    CK(launch_finish_k(g, r->K, hist, r->stream));
+    const int64_t rows = (int64_t)g.lnz * r->ny;
+    int64_t *counts = nullptr, *row_off = nullptr;
+    if ((rc = dmalloc(r, (void **)&counts, (size_t)(rows + 1) * 8))) return rc;
+    if ((rc = dmalloc(r, (void **)&row_off, (size_t)(rows + 1) * 8))) return rc;
+    CK(cudaMemsetAsync(counts, 0, (size_t)(rows + 1) * 8, r->stream));
+    CK(launch_row_counts64(g, r->K, counts, r->stream));
+    size_t tmpb = 0;
+    CK(exclusive_scan_rows64(counts, row_off, rows + 1, nullptr, &tmpb, r->stream));
+    void *tmp = nullptr;
+    if ((rc = dmalloc(r, &tmp, tmpb))) return rc;
+    CK(exclusive_scan_rows64(counts, row_off, rows + 1, tmp, &tmpb, r->stream));
+    unsigned long long h[8];
+    CK(cudaMemcpyAsync(h, hist, sizeof h, cudaMemcpyDeviceToHost, r->stream));
+    CK(cudaMemcpyAsync(&r->nb, row_off + rows, 8, cudaMemcpyDeviceToHost, r->stream));
+    CK(cudaStreamSynchronize(r->stream));
+    r->isolated = (int64_t)h[0];
+    int64_t nin = 0;
+    for (int k = 1; k <= 6; k++) {
+        r->k_hist[k] = (int64_t)h[k];
+        nin += (int64_t)h[k];
+    }
+    r->n_inside = nin;
+    r->k_hist[0] = (int64_t)g.lnz * nxny - nin;
+
+    const int64_t nb = r->nb;
+    if ((rc = dmalloc(r, &r->bpos, (size_t)nb * (r->idx64 ? 8 : 4)))) return rc;
+    if ((rc = dmalloc(r, (void **)&r->bidx, (size_t)nb * 8))) return rc;
+    if ((rc = dmalloc(r, (void **)&r->Kb, (size_t)nb))) return rc;
+    if ((rc = dmalloc(r, (void **)&r->matb, (size_t)nb))) return rc;
+    if ((rc = dmalloc(r, &r->ub, (size_t)nb * sizeof(T)))) return rc;
+    if ((rc = dmalloc(r, &r->gst, (size_t)nb * r->MB * sizeof(T)))) return rc;
+    if ((rc = dmalloc(r, &r->vst, (size_t)nb * r->MB * sizeof(T)))) return rc;
+    CK(cudaMemsetAsync(r->ub, 0, (size_t)nb * sizeof(T) + 16, r->stream));
+    CK(cudaMemsetAsync(r->gst, 0, (size_t)nb * r->MB * sizeof(T) + 16, r->stream));
+    CK(cudaMemsetAsync(r->vst, 0, (size_t)nb * r->MB * sizeof(T) + 16, r->stream));
+    CK(launch_compact(g, r->K, row_off, r->z0, r->ny, r->nx, r->idx64, r->bpos, r->bidx, r->Kb, r->stream));
+
+    // material ids at the boundary nodes (reading R4)
+    unsigned *bad = (unsigned *)(hist + 8);
+    if (!d->matmap) {
+        CK(cudaMemsetAsync(r->matb, 0, (size_t)nb + 1, r->stream));
+    } else if (is_device_ptr(d->matmap)) {
+        CK(launch_gather_mat(d->matmap, (int64_t)mz0 * nxny, r->bidx, 0, nb, r->matb, r->M, bad, r->stream));
+    } else {
+        std::vector<int64_t> off_h((size_t)rows + 1);
+        CK(cudaMemcpyAsync(off_h.data(), row_off, (size_t)(rows + 1) * 8, cudaMemcpyDeviceToHost, r->stream));
+        CK(cudaStreamSynchronize(r->stream));
+        rc = for_plane_chunks(r, d->matmap, mz0, false, (size_t)nxny, r->z0, g.lnz, staging, kStagingBytes,
+                              [&](const void *chunk, int zg, int n) -> int {
+                                  const int64_t i_lo = off_h[(size_t)(zg - r->z0) * r->ny];
+                                  const int64_t i_hi = off_h[(size_t)(zg - r->z0 + n) * r->ny];
+                                  CK(launch_gather_mat((const uint8_t *)chunk, (int64_t)zg * nxny, r->bidx,
+                                                       i_lo, i_hi, r->matb, r->M, bad, r->stream));
+                                  return RAFD_OK;
+                              });
+        if (rc) return rc;
+    }
+    unsigned bad_h = 0;
+    CK(cudaMemcpyAsync(&bad_h, bad, sizeof bad_h, cudaMemcpyDeviceToHost, r->stream));
+    CK(cudaStreamSynchronize(r->stream));
+    cudaFree(hist);
+    cudaFree(counts);
+    cudaFree(row_off);
+    cudaFree(tmp);
+    if (staging) cudaFree(staging);
+    r->device_bytes -= (int64_t)(8 * sizeof(unsigned long long) + sizeof(unsigned)) + 2 * (rows + 1) * 8 +
+                       (int64_t)(tmpb ? tmpb : 16) + (staging ? (int64_t)kStagingBytes : 0);
+    if (bad_h) return set_err(RAFD_E_MATERIAL, "matmap holds a material id >= n_materials (%d) at a boundary node", r->M);
+
+    // ---- tables, control block
+    std::vector<T> tab;
+    std::vector<double> DF;
+    build_tables<T>(d->mat, tab, DF);
+    if ((rc = dmalloc(r, &r->tab, tab.size() * sizeof(T)))) return rc;
+    if ((rc = dmalloc(r, (void **)&r->DF, DF.size() * sizeof(double)))) return rc;
+    CK(cudaMemcpy(r->tab, tab.data(), tab.size() * sizeof(T), cudaMemcpyHostToDevice));
+    CK(cudaMemcpy(r->DF, DF.data(), DF.size() * sizeof(double), cudaMemcpyHostToDevice));
+    if ((rc = dmalloc(r, &r->ctl, sizeof(Ctl<T>)))) return rc;
+    Ctl<T> c{};
+    c.src_pos = -1;
+    CK(cudaMemcpy(r->ctl, &c, sizeof c, cudaMemcpyHostToDevice));
+    return RAFD_OK;
+}
+
+extern "C" int rafd_create(const rafd_room_desc *d, rafd_room **out)
+{
+    if (!out) return set_err(RAFD_E_INVAL, "null out");
+    *out = nullptr;
+    int rc = validate(d);
+    if (rc) return rc;
+    int ndev = 0;
+    if (cudaGetDeviceCount(&ndev) != cudaSuccess || ndev == 0) {
+        cudaGetLastError();
+        return set_err(RAFD_E_CUDA, "no CUDA device (there is no CPU fallback)");
+    }
+    if (d->device < 0 || d->device >= ndev) return set_err(RAFD_E_INVAL, "device %d out of range", d->device);
+    CK(cudaSetDevice(d->device));
+    rafd_room *r = new rafd_room();
+    r->device = d->device;
+    r->prec = d->precision;
+    r->s = d->precision == 32 ? 4 : 8;
+    r->M = d->mat->n_materials;
+    r->MB = d->mat->n_branches;
+    r->nx = d->nx;
+    r->ny = d->ny;
+    r->nz = d->nz;
+    r->lambda = d->lambda;
+    r->rank = d->nranks > 1 ? d->rank : 0;
+    r->nranks = d->nranks > 1 ? d->nranks : 1;
+    r->z0 = r->nranks > 1 ? d->z_begin : 0;
+    r->z1 = r->nranks > 1 ? d->z_end : d->nz;
+    cudaDeviceGetAttribute(&r->nsm, cudaDevAttrMultiProcessorCount, r->device);
+    if (d->cuda_stream) {
+        r->stream = (cudaStream_t)d->cuda_stream;
+    } else {
+        cudaError_t e = cudaStreamCreateWithFlags(&r->stream, cudaStreamNonBlocking);
+        if (e != cudaSuccess) {
+            delete r;
+            return set_err(RAFD_E_CUDA, "cudaStreamCreate: %s", cudaGetErrorString(e));
+        }
+        r->own_stream = true;
+    }
+    cudaStreamCreateWithFlags(&r->cap_stream, cudaStreamNonBlocking);
+    rc = r->prec == 32 ? create_t<float>(r, d) : create_t<double>(r, d);
+    if (!rc && r->nranks > 1) {
+        rc = halo_create(&r->halo, d->nccl_id, r->rank, r->nranks, r->stream);
+        if (rc) set_err(rc, "%s", halo_last_error());
+    }
+    if (rc) {
+        std::string keep = g_err;
+        rafd_destroy(r);
+        g_err = keep;
+        return rc;
+    }
+    *out = r;
+    return RAFD_OK;
+}
+
+static void free_graphs(rafd_room *r)
+{
+    for (int p = 0; p < 2; p++)
+        if (r->graph[p]) {
+            cudaGraphExecDestroy(r->graph[p]);
+            r->graph[p] = nullptr;
+        }
+}
+
+extern "C" void rafd_destroy(rafd_room *r)
+{
+    if (!r) return;
+    cudaSetDevice(r->device);
+    if (r->stream) cudaStreamSynchronize(r->stream);
+    free_graphs(r);
+    if (r->halo) halo_destroy(r->halo);
+    void *ps[] = {r->u[0], r->u[1], r->K, r->bpos, r->bidx, r->Kb, r->matb, r->ub, r->gst, r->vst,
+                  r->tab, r->DF, r->ctl, r->sig, r->rcv_pos, r->rec};
+    for (void *p : ps)
+        if (p) cudaFree(p);
+    for (auto &e : r->evs) {
+        cudaEventDestroy(e.a);
+        cudaEventDestroy(e.b);
+    }
+    for (auto e : r->ev_pool) cudaEventDestroy(e);
+    if (r->cap_stream) cudaStreamDestroy(r->cap_stream);
+    if (r->own_stream && r->stream) cudaStreamDestroy(r->stream);
+    cudaGetLastError();
+    delete r;
+}
+
+// ------------------------------------------------------------------ source / receivers
+static bool owns_plane(const rafd_room *r, int z) { return z >= r->z0 && z < r->z1; }
+
+static int64_t pad_pos(const rafd_room *r, int x, int y, int z)
+{
+    return (int64_t)(z - r->z0 + 1) * r->g.plane + (int64_t)(y + 1) * r->g.pitch + r->g.xo + x;
+}
+
+static int k_at(rafd_room *r, int64_t p, uint8_t *k)
+{
+    CK(cudaStreamSynchronize(r->stream));
+    CK(cudaMemcpy(k, r->K + p, 1, cudaMemcpyDeviceToHost));
+    return RAFD_OK;
+}
+
+template <typename T> static int push_ctl(rafd_room *r, const Ctl<T> &c)
+{
+    CK(cudaStreamSynchronize(r->stream));
+    CK(cudaMemcpy(r->ctl, &c, sizeof c, cudaMemcpyHostToDevice));
+    return RAFD_OK;
+}
+
+template <typename T> static int pull_ctl(rafd_room *r, Ctl<T> &c)
+{
+    CK(cudaStreamSynchronize(r->stream));
+    CK(cudaMemcpy(&c, r->ctl, sizeof c, cudaMemcpyDeviceToHost));
+    return RAFD_OK;
+}
+
+template <typename T>
+static int set_source_t(rafd_room *r, int32_t x, int32_t y, int32_t z, const double *sig, int64_t len)
+{
+    Ctl<T> c;
+    int rc = pull_ctl<T>(r, c);
+    if (rc) return rc;
+    if (r->sig) {
+        cudaFree(r->sig);
+        r->sig = nullptr;
+    }
+    c.sig = nullptr;
+    c.sig_len = 0;
+    c.src_pos = -1;
+    if (len > 0 && owns_plane(r, z)) {
+        const int64_t p = pad_pos(r, x, y, z);
+        uint8_t k = 0;
+        if ((rc = k_at(r, p, &k))) return rc;
+        if (k == 0) return set_err(RAFD_E_OUTSIDE, "source (%d,%d,%d) is at an outside voxel", x, y, z);
+        std::vector<T> st((size_t)len);
+        for (int64_t i = 0; i < len; i++) st[(size_t)i] = (T)sig[i];
+        CK(cudaMalloc(&r->sig, (size_t)len * sizeof(T)));
+        CK(cudaMemcpy(r->sig, st.data(), (size_t)len * sizeof(T), cudaMemcpyHostToDevice));
+        c.sig = (const T *)r->sig;
+        c.sig_len = len;
+        c.src_pos = p;
+    }
+    return push_ctl<T>(r, c);
+}
+
+extern "C" int rafd_set_source(rafd_room *r, int32_t x, int32_t y, int32_t z, const double *sig, int64_t len)
+{
+    if (!r || len < 0 || (len > 0 && !sig)) return set_err(RAFD_E_INVAL, "bad source arguments");
+    if (x < 0 || y < 0 || z < 0 || x >= r->nx || y >= r->ny || z >= r->nz)
+        return set_err(RAFD_E_OUTSIDE, "source (%d,%d,%d) outside the grid", x, y, z);
+    CK(cudaSetDevice(r->device));
+    return r->prec == 32 ? set_source_t<float>(r, x, y, z, sig, len) : set_source_t<double>(r, x, y, z, sig, len);
+}
+
+template <typename T> static int set_receivers_t(rafd_room *r, int32_t n, const int32_t *xyz)
+{
+    std::vector<int64_t> pos((size_t)n);
+    for (int j = 0; j < n; j++) {
+        const int x = xyz[3 * j], y = xyz[3 * j + 1], z = xyz[3 * j + 2];
+        if (x < 0 || y < 0 || z < 0 || x >= r->nx || y >= r->ny || z >= r->nz)
+            return set_err(RAFD_E_OUTSIDE, "receiver %d (%d,%d,%d) outside the grid", j, x, y, z);
+        if (!owns_plane(r, z)) {
+            pos[(size_t)j] = 0;  // padded element 0 is a halo corner: always +0
+            continue;
+        }
+        pos[(size_t)j] = pad_pos(r, x, y, z);
+        uint8_t k = 0;
+        int rc = k_at(r, pos[(size_t)j], &k);
+        if (rc) return rc;
+        if (k == 0) return set_err(RAFD_E_OUTSIDE, "receiver %d (%d,%d,%d) is at an outside voxel", j, x, y, z);
+    }
+    Ctl<T> c;
+    int rc = pull_ctl<T>(r, c);
+    if (rc) return rc;
+    if (r->rcv_pos) cudaFree(r->rcv_pos);
+    if (r->rec) cudaFree(r->rec);
+    r->rcv_pos = nullptr;
+    r->rec = nullptr;
+    r->rec_cap = r->rec_count = 0;
+    r->nrcv = n;
+    if (n > 0) {
+        CK(cudaMalloc((void **)&r->rcv_pos, (size_t)n * 8));
+        CK(cudaMemcpy(r->rcv_pos, pos.data(), (size_t)n * 8, cudaMemcpyHostToDevice));
+    }
+    c.rcv_pos = r->rcv_pos;
+    c.nrcv = n;
+    c.rec = nullptr;
+    c.rec_cap = 0;
+    c.rec_count = 0;
+    return push_ctl<T>(r, c);
+}
+
+extern "C" int rafd_set_receivers(rafd_room *r, int32_t n, const int32_t *xyz)
+{
+    if (!r || n < 0 || (n > 0 && !xyz)) return set_err(RAFD_E_INVAL, "bad receiver arguments");
+    CK(cudaSetDevice(r->device));
+    return r->prec == 32 ? set_receivers_t<float>(r, n, xyz) : set_receivers_t<double>(r, n, xyz);
+}
+
+// grow the receiver buffer so that `more` further steps fit
+template <typename T> static int ensure_rec(rafd_room *r, int64_t more)
+{
+    if (r->nrcv == 0 || r->rec_count + more <= r->rec_cap) return RAFD_OK;
+    int64_t cap = std::max<int64_t>(1024, r->rec_cap * 2);
+    while (cap < r->rec_count + more) cap *= 2;
+    void *nb = nullptr;
+    CK(cudaStreamSynchronize(r->stream));
+    CK(cudaMalloc(&nb, (size_t)cap * r->nrcv * sizeof(T)));
+    if (r->rec && r->rec_count)
+        CK(cudaMemcpy(nb, r->rec, (size_t)r->rec_count * r->nrcv * sizeof(T), cudaMemcpyDeviceToDevice));
+    if (r->rec) cudaFree(r->rec);
+    r->rec = nb;
+    r->rec_cap = cap;
+    Ctl<T> c;
+    int rc = pull_ctl<T>(r, c);
+    if (rc) return rc;
+    c.rec = (T *)nb;
+    c.rec_cap = cap;
+    return push_ctl<T>(r, c);
+}
+
+// ------------------------------------------------------------------ stepping
+template <typename T> static cudaError_t enqueue_step(rafd_room *r, int cur, cudaStream_t s, bool prof)
+{
+    const Grid &g = r->g;
+    T *uc = (T *)r->u[cur];
+    T *un = (T *)r->u[cur ^ 1];
+    auto timed = [&](int kind, auto fn) -> cudaError_t {
+        if (!prof) return fn();
+        cudaEvent_t a, b;
+        if (r->ev_pool.size() >= 2) {
+            a = r->ev_pool.back();
+            r->ev_pool.pop_back();
+            b = r->ev_pool.back();
+            r->ev_pool.pop_back();
+        } else {
+            cudaEventCreate(&a);
+            cudaEventCreate(&b);
+        }
+        cudaEventRecord(a, s);
+        cudaError_t e = fn();
+        cudaEventRecord(b, s);
+        r->evs.push_back({kind, a, b});
+        return e;
+    };
+    cudaError_t e = timed(0, [&] { return launch_volume<T>(g, uc, un, r->K, r->lambda, 0, g.lnz, s); });
+    if (e != cudaSuccess) return e;
+    if (r->nb > 0) {
+        e = timed(1, [&] {
+            return launch_boundary<T>(r->MB, r->idx64, r->bpos, r->Kb, r->matb, 0, r->nb, r->nb, un, uc,
+                                      (T *)r->ub, (T *)r->gst, (T *)r->vst, (const T *)r->tab, r->M,
+                                      r->lambda, s);
+        });
+        if (e != cudaSuccess) return e;
+    }
+    e = timed(2, [&] { return launch_src_rcv<T>(un, ctl_of<T>(r), s); });
+    if (e != cudaSuccess) return e;
+    if (r->halo) {
+        e = halo_exchange(r->halo, un, (size_t)g.plane * sizeof(T), g.lnz, s);
+        if (e != cudaSuccess) return e;
+    }
+    return cudaSuccess;
+}
+
+static int kernels_per_step(const rafd_room *r) { return 2 + (r->nb > 0 ? 1 : 0); }
+
+template <typename T> static int build_graph(rafd_room *r, int parity)
+{
+    cudaGraph_t gr;
+    CK(cudaStreamBeginCapture(r->cap_stream, cudaStreamCaptureModeThreadLocal));
+    cudaError_t e = cudaSuccess;
+    for (int k = 0; k < rafd_room::G && e == cudaSuccess; k++)
+        e = enqueue_step<T>(r, parity ^ (k & 1), r->cap_stream, false);
+    cudaError_t e2 = cudaStreamEndCapture(r->cap_stream, &gr);
+    if (e != cudaSuccess) return set_err(RAFD_E_CUDA, "capture: %s", cudaGetErrorString(e));
+    CK(e2);
+    CK(cudaGraphInstantiate(&r->graph[parity], gr, 0));
+    cudaGraphDestroy(gr);
+    return RAFD_OK;
+}
+
+template <typename T> static int step_t(rafd_room *r, int64_t nsteps)
+{
+    int rc = ensure_rec<T>(r, nsteps);
+    if (rc) return rc;
+    const int kps = kernels_per_step(r);
+    int64_t done = 0;
+    const bool use_graph = !r->profiling && !r->halo && nsteps >= rafd_room::G;
+    while (use_graph && nsteps - done >= rafd_room::G) {
+        if (!r->graph[r->cur] && (rc = build_graph<T>(r, r->cur))) return rc;
+        CK(cudaGraphLaunch(r->graph[r->cur], r->stream));
+        done += rafd_room::G;  // G is even: parity unchanged
+        r->launches += (int64_t)kps * rafd_room::G;
+    }
+    for (; done < nsteps; done++) {
+        cudaError_t e = enqueue_step<T>(r, r->cur, r->stream, r->profiling);
+        if (e != cudaSuccess) return set_err(e == cudaErrorUnknown ? RAFD_E_NCCL : RAFD_E_CUDA, "step: %s", cudaGetErrorString(e));
+        r->cur ^= 1;
+        r->launches += kps;
+    }
+    r->steps += nsteps;
+    if (r->nrcv > 0) r->rec_count += nsteps;
+    return RAFD_OK;
+}
+
+extern "C" int rafd_step(rafd_room *r, int64_t nsteps)
+{
+    if (!r || nsteps < 0) return set_err(RAFD_E_INVAL, "bad step arguments");
+    if (nsteps == 0) return RAFD_OK;
+    CK(cudaSetDevice(r->device));
+    return r->prec == 32 ? step_t<float>(r, nsteps) : step_t<double>(r, nsteps);
+}
+
+extern "C" int rafd_synchronize(rafd_room *r)
+{
+    if (!r) return set_err(RAFD_E_INVAL, "null room");
+    CK(cudaSetDevice(r->device));
+    CK(cudaStreamSynchronize(r->stream));
+    return RAFD_OK;
+}
+
+// ------------------------------------------------------------------ reads
+template <typename T> static int read_receivers_t(rafd_room *r, double *out, int64_t cap, int64_t *nw)
+{
+    CK(cudaStreamSynchronize(r->stream));
+    const int64_t n = r->rec_count;
+    if (r->nrcv > 0 && (cap < n || !out)) return set_err(RAFD_E_INVAL, "cap (%lld) < unread samples (%lld)", (long long)cap, (long long)n);
+    if (r->nrcv > 0 && n > 0) {
+        std::vector<T> h((size_t)n * r->nrcv);
+        CK(cudaMemcpy(h.data(), r->rec, h.size() * sizeof(T), cudaMemcpyDeviceToHost));
+        for (int j = 0; j < r->nrcv; j++)
+            for (int64_t k = 0; k < n; k++) out[j * cap + k] = (double)h[(size_t)k * r->nrcv + j];
+    }
+    *nw = r->nrcv > 0 ? n : 0;
+    r->rec_count = 0;
+    Ctl<T> c;
+    int rc = pull_ctl<T>(r, c);
+    if (rc) return rc;
+    c.rec_count = 0;
+    return push_ctl<T>(r, c);
+}
+
+extern "C" int rafd_read_receivers(rafd_room *r, double *out, int64_t cap, int64_t *n_written)
+{
+    if (!r || !n_written) return set_err(RAFD_E_INVAL, "bad arguments");
+    CK(cudaSetDevice(r->device));
+    return r->prec == 32 ? read_receivers_t<float>(r, out, cap, n_written)
+                         : read_receivers_t<double>(r, out, cap, n_written);
+}
+
+template <typename T> static int field_out_t(rafd_room *r, const T *src, void *dst)
+{
+    const bool dev = is_device_ptr(dst);
+    const size_t pb = (size_t)r->nx * r->ny * sizeof(T);
+    const int lnz = r->g.lnz;
+    if (dev) {
+        CK(launch_field_out<T>(r->g, src, 1, lnz, (T *)dst, r->stream));
+        CK(cudaStreamSynchronize(r->stream));
+        return RAFD_OK;
+    }
+    void *st = nullptr;
+    CK(cudaMalloc(&st, kStagingBytes));
+    const int per = (int)std::max<size_t>(1, kStagingBytes / pb);
+    for (int z = 0; z < lnz; z += per) {
+        const int n = std::min(per, lnz - z);
+        cudaError_t e = launch_field_out<T>(r->g, src, 1 + z, n, (T *)st, r->stream);
+        if (e == cudaSuccess) e = cudaMemcpyAsync((char *)dst + (size_t)z * pb, st, (size_t)n * pb, cudaMemcpyDeviceToHost, r->stream);
+        if (e == cudaSuccess) e = cudaStreamSynchronize(r->stream);
+        if (e != cudaSuccess) {
+            cudaFree(st);
+            return set_err(RAFD_E_CUDA, "read_field: %s", cudaGetErrorString(e));
+        }
+    }
+    cudaFree(st);
+    return RAFD_OK;
+}
+
+extern "C" int rafd_read_field(rafd_room *r, void *u_curr, void *u_prev)
+{
+    if (!r) return set_err(RAFD_E_INVAL, "null room");
+    CK(cudaSetDevice(r->device));
+    int rc = RAFD_OK;
+    if (u_curr) rc = r->prec == 32 ? field_out_t<float>(r, (const float *)r->u[r->cur], u_curr)
+                                   : field_out_t<double>(r, (const double *)r->u[r->cur], u_curr);
+    if (!rc && u_prev) rc = r->prec == 32 ? field_out_t<float>(r, (const float *)r->u[r->cur ^ 1], u_prev)
+                                          : field_out_t<double>(r, (const double *)r->u[r->cur ^ 1], u_prev);
+    return rc;
+}
+
+extern "C" int rafd_read_branch_state(rafd_room *r, void *v, void *g)
+{
+    if (!r) return set_err(RAFD_E_INVAL, "null room");
+    CK(cudaSetDevice(r->device));
+    CK(cudaStreamSynchronize(r->stream));
+    const size_t n = (size_t)r->nb * r->MB * r->s;
+    if (n == 0) return RAFD_OK;
+    if (v) CK(cudaMemcpy(v, r->vst, n, cudaMemcpyDefault));
+    if (g) CK(cudaMemcpy(g, r->gst, n, cudaMemcpyDefault));
+    return RAFD_OK;
+}
+
+extern "C" int rafd_get_classification(rafd_room *r, uint8_t *K, int64_t *bidx, uint8_t *Kb, uint8_t *matb)
+{
+    if (!r) return set_err(RAFD_E_INVAL, "null room");
+    CK(cudaSetDevice(r->device));
+    CK(cudaStreamSynchronize(r->stream));
+    if (K) {
+        const size_t pb = (size_t)r->nx * r->ny;
+        uint8_t *st = nullptr;
+        CK(cudaMalloc((void **)&st, pb * r->g.lnz + 16));
+        CK(launch_field_out<uint8_t>(r->g, r->K, 1, r->g.lnz, st, r->stream));
+        CK(cudaMemcpyAsync(K, st, pb * r->g.lnz, cudaMemcpyDefault, r->stream));
+        CK(cudaStreamSynchronize(r->stream));
+        cudaFree(st);
+    }
+    if (r->nb > 0) {
+        if (bidx) CK(cudaMemcpy(bidx, r->bidx, (size_t)r->nb * 8, cudaMemcpyDefault));
+        if (Kb) CK(cudaMemcpy(Kb, r->Kb, (size_t)r->nb, cudaMemcpyDefault));
+        if (matb) CK(cudaMemcpy(matb, r->matb, (size_t)r->nb, cudaMemcpyDefault));
+    }
+    return RAFD_OK;
+}
+
+// ------------------------------------------------------------------ state in
+template <typename T> static int field_in_t(rafd_room *r, const void *src, T *dst)
+{
+    // planes [z0-1, z1] of the room (ghost planes included when they exist)
+    const bool dev = is_device_ptr(src);
+    const size_t pb = (size_t)r->nx * r->ny * sizeof(T);
+    const int zlo = std::max(0, r->z0 - 1), zhi = std::min(r->nz, r->z1 + 1);
+    void *st = nullptr;
+    if (!dev) CK(cudaMalloc(&st, kStagingBytes));
+    int rc = for_plane_chunks(r, src, 0, dev, pb, zlo, zhi - zlo, st, kStagingBytes,
+                              [&](const void *chunk, int zg, int n) -> int {
+                                  CK(launch_field_in<T>(r->g, (const T *)chunk, zg - r->z0 + 1, n, r->K, dst, r->stream));
+                                  return RAFD_OK;
+                              });
+    cudaStreamSynchronize(r->stream);
+    if (st) cudaFree(st);
+    return rc;
+}
+
+extern "C" int rafd_set_state(rafd_room *r, const void *u_prev, const void *u_curr, const void *v, const void *g)
+{
+    if (!r) return set_err(RAFD_E_INVAL, "null room");
+    CK(cudaSetDevice(r->device));
+    CK(cudaStreamSynchronize(r->stream));
+    int rc = RAFD_OK;
+    if (u_prev) {
+        rc = r->prec == 32 ? field_in_t<float>(r, u_prev, (float *)r->u[r->cur ^ 1])
+                           : field_in_t<double>(r, u_prev, (double *)r->u[r->cur ^ 1]);
+        if (rc) return rc;
+        // ub_prev = u^{n-1} at the boundary nodes (reading R8)
+        if (r->prec == 32) CK(launch_gather_ub<float>(r->bpos, r->idx64, r->nb, (const float *)r->u[r->cur ^ 1], (float *)r->ub, r->stream));
+        else CK(launch_gather_ub<double>(r->bpos, r->idx64, r->nb, (const double *)r->u[r->cur ^ 1], (double *)r->ub, r->stream));
+    }
+    if (u_curr) {
+        rc = r->prec == 32 ? field_in_t<float>(r, u_curr, (float *)r->u[r->cur])
+                           : field_in_t<double>(r, u_curr, (double *)r->u[r->cur]);
+        if (rc) return rc;
+    }
+    const size_t n = (size_t)r->nb * r->MB * r->s;
+    if (n) {
+        if (v) CK(cudaMemcpy(r->vst, v, n, cudaMemcpyDefault));
+        if (g) CK(cudaMemcpy(r->gst, g, n, cudaMemcpyDefault));
+    }
+    CK(cudaStreamSynchronize(r->stream));
+    return RAFD_OK;
+}
+
+// ------------------------------------------------------------------ info / energy / profiling
+static void bytes_per_step(const rafd_room *r, int64_t *vol, int64_t *bnd)
+{
+    // B_step = N_mask*1 + N_in*3s + Nb*(6 + 3s + 4s*MB)
+    const int64_t s = (int64_t)r->s;
+    *vol = (int64_t)r->g.lnz * r->nx * r->ny + r->n_inside * 3 * s;
+    *bnd = r->nb * (6 + 3 * s + 4 * s * r->MB);
+}
+
+extern "C" int rafd_get_info(rafd_room *r, rafd_info *info)
+{
+    if (!r || !info) return set_err(RAFD_E_INVAL, "bad arguments");
+    memset(info, 0, sizeof *info);
+    info->n_mask = (int64_t)r->g.lnz * r->nx * r->ny;
+    info->n_inside = r->n_inside;
+    info->n_boundary = r->nb;
+    for (int k = 0; k < 7; k++) info->k_hist[k] = r->k_hist[k];
+    info->isolated = r->isolated;
+    info->steps = r->steps;
+    bytes_per_step(r, &info->volume_bytes, &info->boundary_bytes);
+    info->bytes_per_step = info->volume_bytes + info->boundary_bytes;
+    info->device_bytes = r->device_bytes;
+    info->precision = r->prec;
+    info->n_materials = r->M;
+    info->n_branches = r->MB;
+    info->z_begin = r->z0;
+    info->z_end = r->z1;
+    info->pitch = (int32_t)r->g.pitch;
+    return RAFD_OK;
+}
+
+extern "C" int rafd_energy(rafd_room *r, double *H)
+{
+    if (!r || !H) return set_err(RAFD_E_INVAL, "bad arguments");
+    CK(cudaSetDevice(r->device));
+    double *acc = nullptr;
+    CK(cudaMalloc((void **)&acc, 3 * sizeof(double)));
+    CK(cudaMemsetAsync(acc, 0, 3 * sizeof(double), r->stream));
+    const void *un1 = r->u[r->cur], *un = r->u[r->cur ^ 1];
+    cudaError_t e;
+    if (r->prec == 32) {
+        e = launch_energy<float>(r->g, (const float *)un1, (const float *)un, r->K, acc, r->stream);
+        if (e == cudaSuccess) e = launch_energy_bnd<float>(r->Kb, r->matb, r->nb, r->MB, (const float *)r->vst, (const float *)r->gst, r->DF, r->M, r->lambda, acc, r->stream);
+    } else {
+        e = launch_energy<double>(r->g, (const double *)un1, (const double *)un, r->K, acc, r->stream);
+        if (e == cudaSuccess) e = launch_energy_bnd<double>(r->Kb, r->matb, r->nb, r->MB, (const double *)r->vst, (const double *)r->gst, r->DF, r->M, r->lambda, acc, r->stream);
+    }
+    double h[3] = {0, 0, 0};
+    if (e == cudaSuccess) e = cudaMemcpyAsync(h, acc, sizeof h, cudaMemcpyDeviceToHost, r->stream);
+    if (e == cudaSuccess) e = cudaStreamSynchronize(r->stream);
+    cudaFree(acc);
+    if (e != cudaSuccess) return set_err(RAFD_E_CUDA, "energy: %s", cudaGetErrorString(e));
+    *H = h[0] + r->lambda * r->lambda * h[1] + h[2];
+    return RAFD_OK;
+}
+
+static void resolve_events(rafd_room *r)
+{
+    if (r->evs.empty()) return;
+    cudaStreamSynchronize(r->stream);
+    for (auto &e : r->evs) {
+        float ms = 0;
+        cudaEventElapsedTime(&ms, e.a, e.b);
+        if (e.kind == 0) {
+            r->kt.volume_ms += ms;
+            r->kt.volume_n++;
+        } else if (e.kind == 1) {
+            r->kt.boundary_ms += ms;
+            r->kt.boundary_n++;
+        } else {
+            r->kt.other_ms += ms;
+            r->kt.other_n++;
+        }
+        r->ev_pool.push_back(e.a);
+        r->ev_pool.push_back(e.b);
+    }
+    r->evs.clear();
+}
+
+extern "C" int rafd_set_profiling(rafd_room *r, int on)
+{
+    if (!r) return set_err(RAFD_E_INVAL, "null room");
+    CK(cudaSetDevice(r->device));
+    resolve_events(r);
+    r->kt = KernelTimes();
+    r->profiling = on != 0;
+    return RAFD_OK;
+}
+
+extern "C" int rafd_get_kernel_times(rafd_room *r, rafd_kernel_times *t)
+{
+    if (!r || !t) return set_err(RAFD_E_INVAL, "bad arguments");
+    CK(cudaSetDevice(r->device));
+    resolve_events(r);
+    t->volume_ms = r->kt.volume_ms;
+    t->boundary_ms = r->kt.boundary_ms;
+    t->other_ms = r->kt.other_ms;
+    t->volume_launches = r->kt.volume_n;
+    t->boundary_launches = r->kt.boundary_n;
+    t->other_launches = r->kt.other_n;
+    return RAFD_OK;
+}
+
+extern "C" int64_t rafd_launch_count(rafd_room *r) { return r ? r->launches : 0; }
+
+// ------------------------------------------------------------------ host-only helpers
+extern "C" int rafd_slab_plan(int32_t nx, int32_t ny, int32_t nz, const uint8_t *mask, int32_t precision,
+                              int32_t n_branches, int32_t nranks, int32_t *z_begin, int32_t *z_end)
+{
+    if (!mask || !z_begin || !z_end || nx < 1 || ny < 1 || nz < 1 || nranks < 1 || nranks > nz)
+        return set_err(RAFD_E_INVAL, "bad slab-plan arguments (need 1 <= nranks <= nz)");
+    if (precision != 32 && precision != 64) return set_err(RAFD_E_INVAL, "precision must be 32 or 64");
+    const int64_t s = precision / 8;
+    const int64_t nxny = (int64_t)nx * ny;
+    // per-plane cost c(z) = N_mask(z) + 3s N_in(z) + (6 + 3s + 4s MB) Nb(z)
+    std::vector<double> cost((size_t)nz);
+    auto in = [&](int64_t x, int64_t y, int64_t z) -> int {
+        if (x < 0 || y < 0 || z < 0 || x >= nx || y >= ny || z >= nz) return 0;
+        return mask[(z * ny + y) * nx + x] ? 1 : 0;
+    };
+    for (int64_t z = 0; z < nz; z++) {
+        int64_t nin = 0, nb = 0;
+        for (int64_t y = 0; y < ny; y++)
+            for (int64_t x = 0; x < nx; x++) {
+                if (!in(x, y, z)) continue;
+                const int k = in(x - 1, y, z) + in(x + 1, y, z) + in(x, y - 1, z) + in(x, y + 1, z) +
+                              in(x, y, z - 1) + in(x, y, z + 1);
+                if (k > 0) nin++;
+                if (k > 0 && k < 6) nb++;
+            }
+        cost[(size_t)z] = (double)nxny + 3.0 * s * nin + (6.0 + 3.0 * s + 4.0 * s * n_branches) * nb;
+    }
+    std::vector<double> pre((size_t)nz + 1, 0.0);
+    for (int z = 0; z < nz; z++) pre[(size_t)z + 1] = pre[(size_t)z] + cost[(size_t)z];
+    const double tot = pre[(size_t)nz];
+    int prev = 0;
+    for (int k = 0; k < nranks; k++) {
+        z_begin[k] = prev;
+        int e;
+        if (k == nranks - 1) {
+            e = nz;
+        } else {
+            const double target = tot * (k + 1) / nranks;
+            e = (int)(std::lower_bound(pre.begin(), pre.end(), target) - pre.begin());
+            // choose the closer cut of the two around the target
+            if (e > 0 && fabs(pre[(size_t)e - 1] - target) <= fabs(pre[(size_t)e] - target)) e -= 1;
+            e = std::max(e, prev + 1);
+            e = std::min(e, nz - (nranks - 1 - k));
+        }
+        z_end[k] = e;
+        prev = e;
+    }
+    return RAFD_OK;
+}
+
+extern "C" int rafd_nccl_unique_id(uint8_t *id128)
+{
+    if (!id128) return set_err(RAFD_E_INVAL, "null id");
+    int rc = halo_unique_id(id128);
+    if (rc) return set_err(rc, "%s", halo_last_error());
+    return RAFD_OK;
+}
+
+extern "C" const char *rafd_last_error(void) { return g_err.c_str(); }
+
+extern "C" const char *rafd_strerror(int code)
+{
+    switch (code) {
+        case RAFD_OK: return "ok";
+        case RAFD_E_INVAL: return "invalid argument";
+        case RAFD_E_UNSTABLE: return "unstable Courant number (lambda^2 > 1/3)";
+        case RAFD_E_NONPASSIVE: return "non-passive boundary material";
+        case RAFD_E_OUTSIDE: return "position outside the room";
+        case RAFD_E_MATERIAL: return "material id out of range";
+        case RAFD_E_NOMEM: return "out of memory";
+        case RAFD_E_CUDA: return "CUDA error";
+        case RAFD_E_NCCL: return "NCCL error";
+        case RAFD_E_STATE: return "invalid state";
+        default: return "unknown error";
+    }
+}
+
+extern "C" int rafd_version(void) { return RAFD_VERSION; }

@@ -262,3 +262,25 @@ def config_materials(cfg):
             return np.asarray(cfg["beta0"], dtype=np.float64), None, None, None
         return fi_beta_from_alpha(C2_ALPHAS[: cfg["M"]]), None, None, None
     return fd_tables(cfg["M"], cfg["MB"])
+
+
+def region_map_box(nx, ny, nz, z_lo, z_hi, M=8, device="cpu"):
+    """The `region` material rule for a BOX room, generated directly for planes
+    [z_lo, z_hi) only (slab-sized inputs for the large halls).  Equals
+    material_map(box_mask(nx, ny, nz), "region", M)[z_lo:z_hi] (tested)."""
+    z = torch.arange(z_lo, z_hi, device=device)[:, None, None]
+    y = torch.arange(ny, device=device)[None, :, None]
+    x = torch.arange(nx, device=device)[None, None, :]
+    shape = (z_hi - z_lo, ny, nx)
+    first = torch.full(shape, 255, dtype=torch.int16, device=device)
+    faces = [z == 0, z == nz - 1, y == 0, y == ny - 1, x == 0, x == nx - 1]
+    for k in range(5, -1, -1):
+        first = torch.where(faces[k].expand(shape), torch.tensor(k, dtype=torch.int16, device=device), first)
+    first = torch.where(first == 255, torch.zeros_like(first), first)
+    if M == 4:
+        lut = torch.tensor([0, 1, 2, 2, 3, 3], dtype=torch.uint8, device=device)
+        return lut[first.long()]
+    out = first.clone()
+    out = torch.where((first == 0) & (x >= nx // 4) & (x < (3 * nx) // 4), torch.tensor(6, dtype=torch.int16, device=device), out)
+    out = torch.where((first >= 2) & (first <= 5) & (z >= (3 * nz) // 4), torch.tensor(7, dtype=torch.int16, device=device), out)
+    return out.to(torch.uint8)

@@ -1,0 +1,319 @@
+"""Thin ctypes binding of librafd.so (include/rafd.h), same names as the C-ABI.
+
+Argument marshalling only: every step of the path runs in the library's CUDA
+kernels.  Buffers may be numpy arrays (host) or torch tensors (host or CUDA);
+the library copies what it needs before a call returns.  There is no CPU
+fallback: loading fails loudly if librafd.so is missing, and rafd_create fails
+with RAFD_E_CUDA when no GPU is present.
+"""
+from __future__ import annotations
+
+import ctypes as C
+import os
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "librafd.so")
+
+RAFD_OK = 0
+RAFD_E_INVAL = -1
+RAFD_E_UNSTABLE = -2
+RAFD_E_NONPASSIVE = -3
+RAFD_E_OUTSIDE = -4
+RAFD_E_MATERIAL = -5
+RAFD_E_NOMEM = -6
+RAFD_E_CUDA = -7
+RAFD_E_NCCL = -8
+RAFD_E_STATE = -9
+
+# every symbol include/rafd.h declares (checked by tests/test_abi.py)
+ABI_SYMBOLS = [
+    "rafd_create", "rafd_destroy", "rafd_set_source", "rafd_set_receivers", "rafd_set_state",
+    "rafd_step", "rafd_synchronize", "rafd_read_receivers", "rafd_read_field",
+    "rafd_read_branch_state", "rafd_get_classification", "rafd_get_info", "rafd_energy",
+    "rafd_set_profiling", "rafd_get_kernel_times", "rafd_launch_count", "rafd_slab_plan",
+    "rafd_nccl_unique_id", "rafd_last_error", "rafd_strerror", "rafd_version",
+]
+
+
+class rafd_materials(C.Structure):
+    _fields_ = [("n_materials", C.c_int32), ("n_branches", C.c_int32),
+                ("beta0", C.c_void_p), ("D", C.c_void_p), ("E", C.c_void_p), ("F", C.c_void_p)]
+
+
+class rafd_room_desc(C.Structure):
+    _fields_ = [("nx", C.c_int32), ("ny", C.c_int32), ("nz", C.c_int32),
+                ("mask", C.c_void_p), ("matmap", C.c_void_p),
+                ("lam", C.c_double), ("precision", C.c_int32),
+                ("mat", C.POINTER(rafd_materials)), ("device", C.c_int32),
+                ("cuda_stream", C.c_void_p), ("rank", C.c_int32), ("nranks", C.c_int32),
+                ("nccl_id", C.c_void_p), ("z_begin", C.c_int32), ("z_end", C.c_int32),
+                ("mask_z0", C.c_int32)]
+
+
+class rafd_info(C.Structure):
+    _fields_ = [("n_mask", C.c_int64), ("n_inside", C.c_int64), ("n_boundary", C.c_int64),
+                ("k_hist", C.c_int64 * 7), ("isolated", C.c_int64), ("steps", C.c_int64),
+                ("bytes_per_step", C.c_int64), ("volume_bytes", C.c_int64),
+                ("boundary_bytes", C.c_int64), ("device_bytes", C.c_int64),
+                ("precision", C.c_int32), ("n_materials", C.c_int32), ("n_branches", C.c_int32),
+                ("z_begin", C.c_int32), ("z_end", C.c_int32), ("pitch", C.c_int32)]
+
+
+class rafd_kernel_times(C.Structure):
+    _fields_ = [("volume_ms", C.c_double), ("boundary_ms", C.c_double), ("other_ms", C.c_double),
+                ("volume_launches", C.c_int64), ("boundary_launches", C.c_int64),
+                ("other_launches", C.c_int64)]
+
+
+_lib = None
+
+
+def lib():
+    """Load librafd.so (raises if it has not been built)."""
+    global _lib
+    if _lib is not None:
+        return _lib
+    if not os.path.exists(LIB_PATH):
+        raise ImportError(f"{LIB_PATH} is missing: build it with "
+                          "`python -m paper_conf_ipps_stoltzfushsld21_b200.build` "
+                          "(there is no CPU fallback)")
+    L = C.CDLL(LIB_PATH)
+    P, I32, I64 = C.c_void_p, C.c_int32, C.c_int64
+    L.rafd_create.argtypes = [C.POINTER(rafd_room_desc), C.POINTER(P)]
+    L.rafd_destroy.argtypes = [P]
+    L.rafd_destroy.restype = None
+    L.rafd_set_source.argtypes = [P, I32, I32, I32, P, I64]
+    L.rafd_set_receivers.argtypes = [P, I32, P]
+    L.rafd_set_state.argtypes = [P, P, P, P, P]
+    L.rafd_step.argtypes = [P, I64]
+    L.rafd_synchronize.argtypes = [P]
+    L.rafd_read_receivers.argtypes = [P, P, I64, C.POINTER(I64)]
+    L.rafd_read_field.argtypes = [P, P, P]
+    L.rafd_read_branch_state.argtypes = [P, P, P]
+    L.rafd_get_classification.argtypes = [P, P, P, P, P]
+    L.rafd_get_info.argtypes = [P, C.POINTER(rafd_info)]
+    L.rafd_energy.argtypes = [P, C.POINTER(C.c_double)]
+    L.rafd_set_profiling.argtypes = [P, C.c_int]
+    L.rafd_get_kernel_times.argtypes = [P, C.POINTER(rafd_kernel_times)]
+    L.rafd_launch_count.argtypes = [P]
+    L.rafd_launch_count.restype = I64
+    L.rafd_slab_plan.argtypes = [I32, I32, I32, P, I32, I32, I32, P, P]
+    L.rafd_nccl_unique_id.argtypes = [P]
+    L.rafd_last_error.restype = C.c_char_p
+    L.rafd_strerror.restype = C.c_char_p
+    L.rafd_strerror.argtypes = [C.c_int]
+    _lib = L
+    return L
+
+
+class RafdError(RuntimeError):
+    def __init__(self, code, msg):
+        super().__init__(f"rafd error {code}: {msg}")
+        self.code = code
+
+
+def _check(rc):
+    if rc != RAFD_OK:
+        raise RafdError(rc, lib().rafd_last_error().decode())
+
+
+def _addr(a):
+    """Address of a numpy array or torch tensor (host or device); None for None."""
+    if a is None:
+        return None
+    if hasattr(a, "data_ptr"):
+        assert a.is_contiguous(), "tensor must be contiguous"
+        return a.data_ptr()
+    assert a.flags["C_CONTIGUOUS"], "array must be C-contiguous"
+    return a.ctypes.data
+
+
+def _f64(a, shape=None):
+    a = np.ascontiguousarray(a, dtype=np.float64)
+    return a if shape is None else a.reshape(shape)
+
+
+class Room:
+    """A room handle (rafd_room*).  Shapes: fields [nz][ny][nx]."""
+
+    def __init__(self, mask, lam, precision, beta0, D=None, E=None, F=None, matmap=None,
+                 device=0, stream=None, rank=0, nranks=1, nccl_id=None, z_begin=0, z_end=0,
+                 mask_z0=0, dims=None):
+        L = lib()
+        # dims = (nx, ny, nz) of the room when `mask` holds only planes [mask_z0, ...)
+        nz, ny, nx = (int(s) for s in mask.shape)
+        if dims is not None:
+            nx, ny, nz = (int(s) for s in dims)
+        beta0 = _f64(beta0).reshape(-1)
+        M = beta0.size
+        if D is None:
+            MB = 0
+            Dd = Ed = Fd = None
+        else:
+            Dd = _f64(D).reshape(M, -1)
+            MB = Dd.shape[1]
+            Ed = _f64(E, (M, MB))
+            Fd = _f64(F, (M, MB))
+        if hasattr(mask, "data_ptr"):
+            assert str(mask.dtype) == "torch.uint8"
+        else:
+            mask = np.ascontiguousarray(mask, dtype=np.uint8)
+        if matmap is not None and not hasattr(matmap, "data_ptr"):
+            matmap = np.ascontiguousarray(matmap, dtype=np.uint8)
+        self._mat = rafd_materials(M, MB, beta0.ctypes.data,
+                                   None if Dd is None else Dd.ctypes.data,
+                                   None if Ed is None else Ed.ctypes.data,
+                                   None if Fd is None else Fd.ctypes.data)
+        idbuf = None
+        if nccl_id is not None:
+            idbuf = (C.c_uint8 * 128).from_buffer_copy(bytes(nccl_id))
+        d = rafd_room_desc(nx, ny, nz, _addr(mask), _addr(matmap), float(lam), int(precision),
+                           C.pointer(self._mat), int(device), stream, int(rank), int(nranks),
+                           None if idbuf is None else C.addressof(idbuf), int(z_begin), int(z_end),
+                           int(mask_z0))
+        h = C.c_void_p()
+        _check(L.rafd_create(C.byref(d), C.byref(h)))
+        self.h = h
+        self._keep = (mask, matmap, beta0, Dd, Ed, Fd)
+        self.shape = (nz, ny, nx)
+        self.precision = int(precision)
+        self.dtype = np.float32 if precision == 32 else np.float64
+        self.M, self.MB = M, MB
+        self.nrcv = 0
+        info = self.get_info()
+        self.z_begin, self.z_end = info["z_begin"], info["z_end"]
+        self.nb = info["n_boundary"]
+
+    # --- lifetime
+    def destroy(self):
+        if getattr(self, "h", None):
+            lib().rafd_destroy(self.h)
+            self.h = None
+
+    def __del__(self):
+        try:
+            self.destroy()
+        except Exception:
+            pass
+
+    # --- set
+    def set_source(self, xyz, sig):
+        sig = _f64(sig).reshape(-1)
+        _check(lib().rafd_set_source(self.h, int(xyz[0]), int(xyz[1]), int(xyz[2]),
+                                     sig.ctypes.data, sig.size))
+
+    def set_receivers(self, xyzs):
+        a = np.ascontiguousarray(np.asarray(xyzs, dtype=np.int32).reshape(-1, 3))
+        _check(lib().rafd_set_receivers(self.h, a.shape[0], a.ctypes.data))
+        self.nrcv = a.shape[0]
+
+    def set_state(self, u_prev=None, u_curr=None, v=None, g=None):
+        def conv(a):
+            if a is None or hasattr(a, "data_ptr"):
+                return a
+            return np.ascontiguousarray(a, dtype=self.dtype)
+        arrs = [conv(a) for a in (u_prev, u_curr, v, g)]
+        _check(lib().rafd_set_state(self.h, *[_addr(a) for a in arrs]))
+
+    # --- run
+    def step(self, n):
+        _check(lib().rafd_step(self.h, int(n)))
+
+    def synchronize(self):
+        _check(lib().rafd_synchronize(self.h))
+
+    # --- read
+    def read_receivers(self, cap=None):
+        if self.nrcv == 0:
+            return np.zeros((0, 0))
+        if cap is None:
+            cap = max(1, self.get_info()["steps"])
+        out = np.zeros((self.nrcv, cap), dtype=np.float64)
+        n = C.c_int64()
+        _check(lib().rafd_read_receivers(self.h, out.ctypes.data, cap, C.byref(n)))
+        return out[:, : n.value].copy()
+
+    def read_field(self, out_curr=None, out_prev=None):
+        """u^n and u^{n-1} of the owned planes (numpy by default; pass CUDA
+        tensors to receive on the device)."""
+        lnz = self.z_end - self.z_begin
+        shp = (lnz, self.shape[1], self.shape[2])
+        cur = np.zeros(shp, dtype=self.dtype) if out_curr is None else out_curr
+        prv = np.zeros(shp, dtype=self.dtype) if out_prev is None else out_prev
+        _check(lib().rafd_read_field(self.h, _addr(cur), _addr(prv)))
+        return cur, prv
+
+    def read_branch_state(self):
+        v = np.zeros((self.MB, self.nb), dtype=self.dtype)
+        g = np.zeros((self.MB, self.nb), dtype=self.dtype)
+        _check(lib().rafd_read_branch_state(self.h, _addr(v), _addr(g)))
+        return v, g
+
+    def get_classification(self):
+        lnz = self.z_end - self.z_begin
+        K = np.zeros((lnz, self.shape[1], self.shape[2]), dtype=np.uint8)
+        bidx = np.zeros(self.nb, dtype=np.int64)
+        Kb = np.zeros(self.nb, dtype=np.uint8)
+        matb = np.zeros(self.nb, dtype=np.uint8)
+        _check(lib().rafd_get_classification(self.h, K.ctypes.data, bidx.ctypes.data,
+                                             Kb.ctypes.data, matb.ctypes.data))
+        return K, bidx, Kb, matb
+
+    def get_info(self):
+        i = rafd_info()
+        _check(lib().rafd_get_info(self.h, C.byref(i)))
+        d = {k: getattr(i, k) for k, _ in rafd_info._fields_}
+        d["k_hist"] = list(i.k_hist)
+        return d
+
+    def energy(self):
+        h = C.c_double()
+        _check(lib().rafd_energy(self.h, C.byref(h)))
+        return h.value
+
+    def set_profiling(self, on=True):
+        _check(lib().rafd_set_profiling(self.h, 1 if on else 0))
+
+    def get_kernel_times(self):
+        t = rafd_kernel_times()
+        _check(lib().rafd_get_kernel_times(self.h, C.byref(t)))
+        return {k: getattr(t, k) for k, _ in rafd_kernel_times._fields_}
+
+    def launch_count(self):
+        return int(lib().rafd_launch_count(self.h))
+
+
+# ------------------------------------------------------------------ C-ABI names
+def rafd_create(*a, **k):
+    return Room(*a, **k)
+
+
+def rafd_destroy(room):
+    room.destroy()
+
+
+def rafd_slab_plan(mask, precision, n_branches, nranks):
+    """Cost-weighted z-slab split (host-only, no GPU).  Returns [(z_begin, z_end)]."""
+    m = np.ascontiguousarray(mask, dtype=np.uint8)
+    nz, ny, nx = m.shape
+    zb = np.zeros(nranks, dtype=np.int32)
+    ze = np.zeros(nranks, dtype=np.int32)
+    _check(lib().rafd_slab_plan(nx, ny, nz, m.ctypes.data, int(precision), int(n_branches),
+                                int(nranks), zb.ctypes.data, ze.ctypes.data))
+    return list(zip(zb.tolist(), ze.tolist()))
+
+
+def rafd_nccl_unique_id():
+    buf = (C.c_uint8 * 128)()
+    _check(lib().rafd_nccl_unique_id(buf))
+    return bytes(buf)
+
+
+def rafd_version():
+    return int(lib().rafd_version())
+
+
+def rafd_strerror(code):
+    return lib().rafd_strerror(int(code)).decode()
