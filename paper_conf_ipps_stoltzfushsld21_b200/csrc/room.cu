@@ -113,9 +113,10 @@ struct rafd_room {
 
 template <typename T> static Ctl<T> *ctl_of(rafd_room *r) { return (Ctl<T> *)r->ctl; }
 
+// every allocation carries 64 bytes of slack (vector loads / memsets of +16)
 static int dmalloc(rafd_room *r, void **p, size_t bytes)
 {
-    if (bytes == 0) bytes = 16;
+    bytes += 64;
     cudaError_t e = cudaMalloc(p, bytes);
     if (e != cudaSuccess) {
         cudaGetLastError();
