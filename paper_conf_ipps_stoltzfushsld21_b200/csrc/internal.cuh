@@ -4,6 +4,7 @@
 #include <cuda_runtime.h>
 #include <stdint.h>
 
+#include <algorithm>
 #include <string>
 #include <vector>
 
@@ -62,9 +63,14 @@ struct KernelTimes {
 
 // ------------------------------------------------------------------ launchers
 // (each returns cudaGetLastError() of its launch)
+// plan == nullptr selects the one-thread-per-voxel v0 kernel (A/B reference);
+// cur_idx = which of the two field buffers holds u^n (selects the TMA maps).
 template <typename T>
 cudaError_t launch_volume(const Grid &g, const T *cur, T *nxt, const uint8_t *K, double lambda,
-                          int z_lo, int z_hi, cudaStream_t s);
+                          int z_lo, int z_hi, cudaStream_t s, const void *plan, int cur_idx);
+template <typename T>
+cudaError_t volume_plan_create(const Grid &g, void *u0, void *u1, uint8_t *K, int nsm, void **plan);
+void volume_plan_destroy(void *plan);
 template <typename T>
 cudaError_t launch_boundary(int MB, bool idx64, const void *bpos, const uint8_t *Kb,
                             const uint8_t *matb, int64_t i_lo, int64_t i_hi, int64_t Nb, T *unext,

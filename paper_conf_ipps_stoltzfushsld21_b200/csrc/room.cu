@@ -13,6 +13,7 @@
 #include <math.h>
 #include <stdarg.h>
 #include <stdio.h>
+#include <stdlib.h>
 #include <string.h>
 
 #include <algorithm>
@@ -74,7 +75,7 @@ struct rafd_room {
     int nsm = 148;
     void *u[2] = {nullptr, nullptr};
     int cur = 0;  // u[cur] = u^n
-    uint8_t *K = nullptr;
+    uint8_t *K = nullptr, *K_alloc = nullptr;
     int64_t nb = 0;
     bool idx64 = false;
     void *bpos = nullptr;
@@ -109,6 +110,8 @@ struct rafd_room {
     KernelTimes kt;
     // multi-GPU halo exchange
     Halo *halo = nullptr;
+    // TMA tensor maps etc. of the volume kernel (nullptr => v0 kernel)
+    void *vplan = nullptr;
 };
 
 template <typename T> static Ctl<T> *ctl_of(rafd_room *r) { return (Ctl<T> *)r->ctl; }
@@ -229,10 +232,14 @@ template <typename T> static int create_t(rafd_room *r, const rafd_room_desc *d)
     r->idx64 = g.total >= (int64_t)UINT32_MAX;
 
     int rc;
-    if ((rc = dmalloc(r, (void **)&r->K, (size_t)g.total + 64))) return rc;
+    // K grid: element (row, xo + x) must sit at a 16-byte aligned byte address
+    // for the TMA boxes of the volume kernel, so the buffer starts 16 - xo bytes
+    // before the first element (r->K_alloc is what cudaMalloc returned).
+    if ((rc = dmalloc(r, (void **)&r->K_alloc, (size_t)g.total + 64))) return rc;
+    r->K = r->K_alloc + (16 - g.xo);
     for (int k = 0; k < 2; k++)
         if ((rc = dmalloc(r, &r->u[k], (size_t)g.total * sizeof(T) + 64))) return rc;
-    CK(cudaMemsetAsync(r->K, 0, (size_t)g.total + 64, r->stream));
+    CK(cudaMemsetAsync(r->K_alloc, 0, (size_t)g.total + 64, r->stream));
     for (int k = 0; k < 2; k++) CK(cudaMemsetAsync(r->u[k], 0, (size_t)g.total * sizeof(T) + 64, r->stream));
 
     // ---- classification (row a1)
@@ -335,6 +342,8 @@ template <typename T> static int create_t(rafd_room *r, const rafd_room_desc *d)
     Ctl<T> c{};
     c.src_pos = -1;
     CK(cudaMemcpy(r->ctl, &c, sizeof c, cudaMemcpyHostToDevice));
+    const char *env = getenv("RAFD_VOLUME_KERNEL");
+    if (!(env && strcmp(env, "v0") == 0)) CK(volume_plan_create<T>(g, r->u[0], r->u[1], r->K_alloc, r->nsm, &r->vplan));
     return RAFD_OK;
 }
 
@@ -408,7 +417,8 @@ extern "C" void rafd_destroy(rafd_room *r)
     if (r->stream) cudaStreamSynchronize(r->stream);
     free_graphs(r);
     if (r->halo) halo_destroy(r->halo);
-    void *ps[] = {r->u[0], r->u[1], r->K, r->bpos, r->bidx, r->Kb, r->matb, r->ub, r->gst, r->vst,
+    if (r->vplan) volume_plan_destroy(r->vplan);
+    void *ps[] = {r->u[0], r->u[1], r->K_alloc, r->bpos, r->bidx, r->Kb, r->matb, r->ub, r->gst, r->vst,
                   r->tab, r->DF, r->ctl, r->sig, r->rcv_pos, r->rec};
     for (void *p : ps)
         if (p) cudaFree(p);
@@ -581,7 +591,7 @@ template <typename T> static cudaError_t enqueue_step(rafd_room *r, int cur, cud
         r->evs.push_back({kind, a, b});
         return e;
     };
-    cudaError_t e = timed(0, [&] { return launch_volume<T>(g, uc, un, r->K, r->lambda, 0, g.lnz, s); });
+    cudaError_t e = timed(0, [&] { return launch_volume<T>(g, uc, un, r->K, r->lambda, 0, g.lnz, s, r->vplan, cur); });
     if (e != cudaSuccess) return e;
     if (r->nb > 0) {
         e = timed(1, [&] {
