@@ -220,3 +220,27 @@ def test_errors(orc):
         g.read_receivers(cap=5)
     assert e.value.code == rafd.RAFD_E_INVAL
     assert g.read_receivers(cap=10).shape == (1, 10)
+
+
+@pytest.mark.parametrize("cfg", [0, 1, 2, 3])
+@pytest.mark.parametrize("precision", [32, 64])
+def test_volume_tile_configs_bitwise(orc, cfg, precision, monkeypatch):
+    """Every tile configuration of the TMA volume kernel (RAFD_VOL_CFG) and the
+    one-thread-per-voxel v0 kernel give the oracle's bits; the room (150x75x40)
+    spans several tiles in x and y with ragged tails."""
+    monkeypatch.setenv("RAFD_VOL_CFG", str(cfg))
+    mask = I.dome_mask(150, 75, 40).numpy()
+    mm = I.material_map(torch.from_numpy(mask), "region", 8).numpy()
+    beta0, D, E, F = I.fd_tables(8, 3)
+    o, g = pair(orc, mask, precision, beta0, D, E, F, matmap=mm)
+    src = I.snap_inside(mask, (70, 30, 20))
+    for r in (o, g):
+        r.set_source(src, I.gaussian_pulse(30, 4.0))
+        r.step(60)
+    assert_close(o.read_field()[0], g.read_field()[0], precision, f"cfg {cfg}")
+    if cfg == 0:
+        monkeypatch.setenv("RAFD_VOLUME_KERNEL", "v0")
+        g0 = rafd.Room(mask, LAM, precision, beta0, D, E, F, matmap=mm)
+        g0.set_source(src, I.gaussian_pulse(30, 4.0))
+        g0.step(60)
+        assert_close(o.read_field()[0], g0.read_field()[0], precision, "v0")
