@@ -82,7 +82,8 @@ typedef struct rafd_room_desc {
      * rafd_slab_plan) and exchanges one halo plane with ranks +-1 every step
      * over NCCL; every rank passes the same mask/matmap/materials. */
     int32_t rank, nranks;
-    const uint8_t *nccl_id;  /* 128-byte ncclUniqueId from rafd_nccl_unique_id (rank 0), or NULL */
+    const uint8_t *nccl_id;  /* 128-byte ncclUniqueId from rafd_nccl_unique_id (rank 0); NULL for */
+                             /* slabs held by one process and stepped with rafd_step_group      */
     int32_t z_begin, z_end;
     /* mask / matmap hold planes [mask_z0, ...) of the room (0: the whole room).
      * A slab handle reads planes [z_begin-1, z_end] (clipped to the room), so a
@@ -144,6 +145,14 @@ int rafd_set_state(rafd_room *r, const void *u_prev, const void *u_curr, const v
 /* Enqueue nsteps time steps (volume kernel, boundary kernel, source,
  * receivers, rotation).  Asynchronous w.r.t. the host. */
 int rafd_step(rafd_room *r, int64_t nsteps);
+
+/* Step the n slabs of one room held by this process (created with nranks = n,
+ * rank = k, nccl_id = NULL, consecutive [z_begin, z_end)), on one or several
+ * devices: per step every slab runs its kernels, then its two ghost planes are
+ * copied from its neighbours (cudaMemcpyPeerAsync, event-ordered).  Results
+ * are bitwise those of the undivided room.  STATE if the handles are not such
+ * a group.  rafd_step on a slab without nccl_id returns STATE. */
+int rafd_step_group(rafd_room **rooms, int32_t n, int64_t nsteps);
 
 /* Wait for all enqueued work of the room. */
 int rafd_synchronize(rafd_room *r);

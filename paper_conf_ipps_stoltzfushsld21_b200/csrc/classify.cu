@@ -15,7 +15,8 @@
 //   count_k      : K[p] = 0x80 | (# of 6 face neighbours with bit 7) for owned
 //                  inside voxels (bit 7 is never changed, so concurrent
 //                  neighbour reads are consistent)
-//   finish_k     : K[p] &= 0x7f on owned planes, histogram; ghost planes -> 0
+//   finish_k     : K[p] &= 0x7f on owned planes, histogram (ghost planes keep
+//                  their 0x80 flags)
 //   row_counts   : boundary nodes per (z, y) row
 //   exclusive scan (CUB) -> row offsets
 //   compact      : per row, a block scan writes the nodes in ascending x
@@ -170,12 +171,10 @@ cudaError_t launch_finish_k(const Grid &g, uint8_t *K, unsigned long long *hist8
 {
     const int64_t n = (int64_t)g.lnz * g.ny * g.nx;
     k_finish_k<<<grid_for(n), 256, 0, s>>>(g, K, hist8);
-    cudaError_t e = cudaGetLastError();
-    if (e != cudaSuccess) return e;
-    // ghost planes carry only neighbour flags; clear them
-    e = cudaMemsetAsync(K, 0, (size_t)g.plane, s);
-    if (e != cudaSuccess) return e;
-    return cudaMemsetAsync(K + (int64_t)(g.lnz + 1) * g.plane, 0, (size_t)g.plane, s);
+    // the two ghost planes keep their 0x80 inside flags: set_state / read use
+    // them to keep ghost values, the energy hook for cross-slab edges; no
+    // kernel of the step reads K there
+    return cudaGetLastError();
 }
 
 cudaError_t launch_row_counts64(const Grid &g, const uint8_t *K, int64_t *counts, cudaStream_t s)

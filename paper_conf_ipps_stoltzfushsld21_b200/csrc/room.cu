@@ -108,8 +108,11 @@ struct rafd_room {
     std::vector<Ev> evs;
     std::vector<cudaEvent_t> ev_pool;
     KernelTimes kt;
-    // multi-GPU halo exchange
+    // multi-GPU halo exchange: NCCL (one rank per process) or, for slabs of one
+    // process (rafd_step_group), device-to-device / peer copies
     Halo *halo = nullptr;
+    bool local_slab = false;
+    cudaEvent_t ev_done = nullptr, ev_copied = nullptr;
     // TMA tensor maps etc. of the volume kernel (nullptr => v0 kernel)
     void *vplan = nullptr;
 };
@@ -388,8 +391,14 @@ extern "C" int rafd_create(const rafd_room_desc *d, rafd_room **out)
     cudaStreamCreateWithFlags(&r->cap_stream, cudaStreamNonBlocking);
     rc = r->prec == 32 ? create_t<float>(r, d) : create_t<double>(r, d);
     if (!rc && r->nranks > 1) {
-        rc = halo_create(&r->halo, d->nccl_id, r->rank, r->nranks, r->stream);
-        if (rc) set_err(rc, "%s", halo_last_error());
+        if (d->nccl_id) {
+            rc = halo_create(&r->halo, d->nccl_id, r->rank, r->nranks, r->stream);
+            if (rc) set_err(rc, "%s", halo_last_error());
+        } else {
+            r->local_slab = true;  // stepped by rafd_step_group in this process
+            cudaEventCreateWithFlags(&r->ev_done, cudaEventDisableTiming);
+            cudaEventCreateWithFlags(&r->ev_copied, cudaEventDisableTiming);
+        }
     }
     if (rc) {
         std::string keep = g_err;
@@ -417,6 +426,8 @@ extern "C" void rafd_destroy(rafd_room *r)
     if (r->stream) cudaStreamSynchronize(r->stream);
     free_graphs(r);
     if (r->halo) halo_destroy(r->halo);
+    if (r->ev_done) cudaEventDestroy(r->ev_done);
+    if (r->ev_copied) cudaEventDestroy(r->ev_copied);
     if (r->vplan) volume_plan_destroy(r->vplan);
     void *ps[] = {r->u[0], r->u[1], r->K_alloc, r->bpos, r->bidx, r->Kb, r->matb, r->ub, r->gst, r->vst,
                   r->tab, r->DF, r->ctl, r->sig, r->rcv_pos, r->rec};
@@ -654,9 +665,94 @@ template <typename T> static int step_t(rafd_room *r, int64_t nsteps)
 extern "C" int rafd_step(rafd_room *r, int64_t nsteps)
 {
     if (!r || nsteps < 0) return set_err(RAFD_E_INVAL, "bad step arguments");
+    if (r->local_slab) return set_err(RAFD_E_STATE, "a slab created without nccl_id is stepped with rafd_step_group");
     if (nsteps == 0) return RAFD_OK;
     CK(cudaSetDevice(r->device));
     return r->prec == 32 ? step_t<float>(r, nsteps) : step_t<double>(r, nsteps);
+}
+
+// Slabs of one room held by this process (one per device, or several on one
+// device): every step, each slab runs its kernels on its own stream, then pulls
+// its two ghost planes from its neighbours' current u buffers (cudaMemcpyAsync,
+// peer copy across devices), ordered by events; a slab's next step waits for
+// its neighbours' copies out of its buffer.  Results are identical to one room.
+template <typename T> static int step_group_t(rafd_room **rs, int n, int64_t nsteps)
+{
+    for (int k = 0; k < n; k++) {
+        int rc = ensure_rec<T>(rs[k], nsteps);
+        if (rc) return rc;
+    }
+    for (int64_t st = 0; st < nsteps; st++) {
+        for (int k = 0; k < n; k++) {
+            rafd_room *r = rs[k];
+            CK(cudaSetDevice(r->device));
+            if (st > 0) {  // neighbours must have finished reading our previous buffer
+                if (k > 0) CK(cudaStreamWaitEvent(r->stream, rs[k - 1]->ev_copied, 0));
+                if (k < n - 1) CK(cudaStreamWaitEvent(r->stream, rs[k + 1]->ev_copied, 0));
+            }
+            cudaError_t e = enqueue_step<T>(r, r->cur, r->stream, r->profiling);
+            if (e != cudaSuccess) return set_err(RAFD_E_CUDA, "step: %s", cudaGetErrorString(e));
+            CK(cudaEventRecord(r->ev_done, r->stream));
+            r->launches += kernels_per_step(r);
+        }
+        for (int k = 0; k < n; k++) {
+            rafd_room *r = rs[k];
+            CK(cudaSetDevice(r->device));
+            const size_t pb = (size_t)r->g.plane * sizeof(T);
+            char *mine = (char *)r->u[r->cur ^ 1];  // u^{n+1} of this slab
+            if (k > 0) {
+                rafd_room *q = rs[k - 1];
+                CK(cudaStreamWaitEvent(r->stream, q->ev_done, 0));
+                const char *src = (const char *)q->u[q->cur ^ 1] + (size_t)q->g.lnz * pb;
+                CK(cudaMemcpyPeerAsync(mine, r->device, src, q->device, pb, r->stream));
+            }
+            if (k < n - 1) {
+                rafd_room *q = rs[k + 1];
+                CK(cudaStreamWaitEvent(r->stream, q->ev_done, 0));
+                const char *src = (const char *)q->u[q->cur ^ 1] + pb;
+                CK(cudaMemcpyPeerAsync(mine + (size_t)(r->g.lnz + 1) * pb, r->device, src, q->device, pb, r->stream));
+            }
+            CK(cudaEventRecord(r->ev_copied, r->stream));
+        }
+        for (int k = 0; k < n; k++) rs[k]->cur ^= 1;
+    }
+    for (int k = 0; k < n; k++) {
+        rs[k]->steps += nsteps;
+        if (rs[k]->nrcv > 0) rs[k]->rec_count += nsteps;
+    }
+    return RAFD_OK;
+}
+
+extern "C" int rafd_step_group(rafd_room **rooms, int32_t n, int64_t nsteps)
+{
+    if (!rooms || n < 1 || nsteps < 0) return set_err(RAFD_E_INVAL, "bad group arguments");
+    for (int k = 0; k < n; k++) {
+        rafd_room *r = rooms[k];
+        if (!r) return set_err(RAFD_E_INVAL, "null room in group");
+        if (n == 1 ? r->nranks != 1 : (!r->local_slab || r->nranks != n || r->rank != k))
+            return set_err(RAFD_E_STATE, "group member %d is not local slab %d of %d", k, k, n);
+        if (r->prec != rooms[0]->prec || r->nx != rooms[0]->nx || r->ny != rooms[0]->ny || r->nz != rooms[0]->nz)
+            return set_err(RAFD_E_STATE, "group members are not slabs of one room");
+        if (k > 0 && rooms[k - 1]->z1 != r->z0) return set_err(RAFD_E_STATE, "slabs are not contiguous");
+    }
+    if (nsteps == 0) return RAFD_OK;
+    if (n == 1) return rafd_step(rooms[0], nsteps);
+    // peer access between distinct devices (best effort; cudaMemcpyPeerAsync works without it)
+    for (int k = 0; k + 1 < n; k++) {
+        const int a = rooms[k]->device, b = rooms[k + 1]->device;
+        if (a != b) {
+            int can = 0;
+            cudaDeviceCanAccessPeer(&can, a, b);
+            if (can) {
+                cudaSetDevice(a);
+                cudaDeviceEnablePeerAccess(b, 0);
+                cudaSetDevice(b);
+                cudaDeviceEnablePeerAccess(a, 0);
+                cudaGetLastError();
+            }
+        }
+    }
+    return rooms[0]->prec == 32 ? step_group_t<float>(rooms, n, nsteps) : step_group_t<double>(rooms, n, nsteps);
 }
 
 extern "C" int rafd_synchronize(rafd_room *r)

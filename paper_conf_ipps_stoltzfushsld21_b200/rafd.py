@@ -30,7 +30,7 @@ RAFD_E_STATE = -9
 # every symbol include/rafd.h declares (checked by tests/test_abi.py)
 ABI_SYMBOLS = [
     "rafd_create", "rafd_destroy", "rafd_set_source", "rafd_set_receivers", "rafd_set_state",
-    "rafd_step", "rafd_synchronize", "rafd_read_receivers", "rafd_read_field",
+    "rafd_step", "rafd_step_group", "rafd_synchronize", "rafd_read_receivers", "rafd_read_field",
     "rafd_read_branch_state", "rafd_get_classification", "rafd_get_info", "rafd_energy",
     "rafd_set_profiling", "rafd_get_kernel_times", "rafd_launch_count", "rafd_slab_plan",
     "rafd_nccl_unique_id", "rafd_last_error", "rafd_strerror", "rafd_version",
@@ -88,6 +88,7 @@ def lib():
     L.rafd_set_receivers.argtypes = [P, I32, P]
     L.rafd_set_state.argtypes = [P, P, P, P, P]
     L.rafd_step.argtypes = [P, I64]
+    L.rafd_step_group.argtypes = [C.POINTER(P), I32, I64]
     L.rafd_synchronize.argtypes = [P]
     L.rafd_read_receivers.argtypes = [P, P, I64, C.POINTER(I64)]
     L.rafd_read_field.argtypes = [P, P, P]
@@ -294,6 +295,12 @@ def rafd_destroy(room):
     room.destroy()
 
 
+def rafd_step_group(rooms, nsteps):
+    """Step the slabs of one room held by this process (see include/rafd.h)."""
+    arr = (C.c_void_p * len(rooms))(*[r.h.value for r in rooms])
+    _check(lib().rafd_step_group(arr, len(rooms), int(nsteps)))
+
+
 def rafd_slab_plan(mask, precision, n_branches, nranks):
     """Cost-weighted z-slab split (host-only, no GPU).  Returns [(z_begin, z_end)]."""
     m = np.ascontiguousarray(mask, dtype=np.uint8)
@@ -303,6 +310,23 @@ def rafd_slab_plan(mask, precision, n_branches, nranks):
     _check(lib().rafd_slab_plan(nx, ny, nz, m.ctypes.data, int(precision), int(n_branches),
                                 int(nranks), zb.ctypes.data, ze.ctypes.data))
     return list(zip(zb.tolist(), ze.tolist()))
+
+
+def slab_owner(z, plan):
+    """Index of the slab of `plan` [(z_begin, z_end)] that owns plane z."""
+    for k, (a, b) in enumerate(plan):
+        if a <= z < b:
+            return k
+    raise ValueError(f"plane {z} outside the plan")
+
+
+def gather_receivers(per_slab, xyzs, plan):
+    """Receiver traces of a slab-decomposed room: row j comes from the slab that
+    owns receiver j's plane (the other slabs record +0 there)."""
+    out = np.zeros_like(per_slab[0])
+    for j, (x, y, z) in enumerate(xyzs):
+        out[j] = per_slab[slab_owner(z, plan)][j]
+    return out
 
 
 def rafd_nccl_unique_id():
