@@ -77,7 +77,7 @@ cudaError_t launch_boundary(int MB, bool idx64, const void *bpos, const uint8_t 
                             const T *ucur, T *ub_prev, T *g, T *v, const T *tab, int M,
                             double lambda, cudaStream_t s);
 template <typename T>
-cudaError_t launch_src_rcv(T *unext, Ctl<T> *ctl, cudaStream_t s);
+cudaError_t launch_src_rcv(T *unext, Ctl<T> *ctl, cudaStream_t s, int mode = 3);
 
 // classification: flags -> K (in place, bit 7 trick), counts, compaction
 cudaError_t launch_scatter_mask(const Grid &g, const uint8_t *mask_chunk, int zp0, int nzc,

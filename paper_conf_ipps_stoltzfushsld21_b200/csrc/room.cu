@@ -112,7 +112,12 @@ struct rafd_room {
     // process (rafd_step_group), device-to-device / peer copies
     Halo *halo = nullptr;
     bool local_slab = false;
-    cudaEvent_t ev_done = nullptr, ev_copied = nullptr;
+    // edge-first step of a slab: edge planes, then the halo exchange on
+    // comm_stream overlapped with the interior planes
+    cudaStream_t comm_stream = nullptr;
+    cudaEvent_t ev_edge = nullptr, ev_halo = nullptr;
+    int64_t n_first_plane = 0, n_last_start = 0;  // node ranges [0, n_first_plane), [n_last_start, nb)
+    int src_z = -1;                                // global plane of the source (-1: none)
     // TMA tensor maps etc. of the volume kernel (nullptr => v0 kernel)
     void *vplan = nullptr;
 };
@@ -278,6 +283,9 @@ template <typename T> static int create_t(rafd_room *r, const rafd_room_desc *d)
     unsigned long long h[8];
     CK(cudaMemcpyAsync(h, hist, sizeof h, cudaMemcpyDeviceToHost, r->stream));
     CK(cudaMemcpyAsync(&r->nb, row_off + rows, 8, cudaMemcpyDeviceToHost, r->stream));
+    // boundary nodes of the first / last owned plane (edge phase of a slab)
+    CK(cudaMemcpyAsync(&r->n_first_plane, row_off + std::min<int64_t>(rows, r->ny), 8, cudaMemcpyDeviceToHost, r->stream));
+    CK(cudaMemcpyAsync(&r->n_last_start, row_off + (int64_t)(g.lnz - 1) * r->ny, 8, cudaMemcpyDeviceToHost, r->stream));
     CK(cudaStreamSynchronize(r->stream));
     r->isolated = (int64_t)h[0];
     int64_t nin = 0;
@@ -396,9 +404,10 @@ extern "C" int rafd_create(const rafd_room_desc *d, rafd_room **out)
             if (rc) set_err(rc, "%s", halo_last_error());
         } else {
             r->local_slab = true;  // stepped by rafd_step_group in this process
-            cudaEventCreateWithFlags(&r->ev_done, cudaEventDisableTiming);
-            cudaEventCreateWithFlags(&r->ev_copied, cudaEventDisableTiming);
         }
+        cudaStreamCreateWithFlags(&r->comm_stream, cudaStreamNonBlocking);
+        cudaEventCreateWithFlags(&r->ev_edge, cudaEventDisableTiming);
+        cudaEventCreateWithFlags(&r->ev_halo, cudaEventDisableTiming);
     }
     if (rc) {
         std::string keep = g_err;
@@ -426,8 +435,9 @@ extern "C" void rafd_destroy(rafd_room *r)
     if (r->stream) cudaStreamSynchronize(r->stream);
     free_graphs(r);
     if (r->halo) halo_destroy(r->halo);
-    if (r->ev_done) cudaEventDestroy(r->ev_done);
-    if (r->ev_copied) cudaEventDestroy(r->ev_copied);
+    if (r->ev_edge) cudaEventDestroy(r->ev_edge);
+    if (r->ev_halo) cudaEventDestroy(r->ev_halo);
+    if (r->comm_stream) cudaStreamDestroy(r->comm_stream);
     if (r->vplan) volume_plan_destroy(r->vplan);
     void *ps[] = {r->u[0], r->u[1], r->K_alloc, r->bpos, r->bidx, r->Kb, r->matb, r->ub, r->gst, r->vst,
                   r->tab, r->DF, r->ctl, r->sig, r->rcv_pos, r->rec};
@@ -486,6 +496,7 @@ static int set_source_t(rafd_room *r, int32_t x, int32_t y, int32_t z, const dou
     c.sig = nullptr;
     c.sig_len = 0;
     c.src_pos = -1;
+    r->src_z = -1;
     if (len > 0 && owns_plane(r, z)) {
         const int64_t p = pad_pos(r, x, y, z);
         uint8_t k = 0;
@@ -498,6 +509,7 @@ static int set_source_t(rafd_room *r, int32_t x, int32_t y, int32_t z, const dou
         c.sig = (const T *)r->sig;
         c.sig_len = len;
         c.src_pos = p;
+        r->src_z = z;
     }
     return push_ctl<T>(r, c);
 }
@@ -614,11 +626,83 @@ template <typename T> static cudaError_t enqueue_step(rafd_room *r, int cur, cud
     }
     e = timed(2, [&] { return launch_src_rcv<T>(un, ctl_of<T>(r), s); });
     if (e != cudaSuccess) return e;
-    if (r->halo) {
-        e = halo_exchange(r->halo, un, (size_t)g.plane * sizeof(T), g.lnz, s);
-        if (e != cudaSuccess) return e;
-    }
     return cudaSuccess;
+}
+
+// ---- slab step, edge planes first: phase 0 = the first and
+// last owned plane (volume, their boundary nodes, the source if it lies there),
+// then the halo exchange runs on comm_stream while phase 1 = the interior
+// planes (volume, boundary nodes, source, receivers) runs on the main stream.
+template <typename T> static cudaError_t enqueue_phase(rafd_room *r, int phase, cudaStream_t s, bool prof)
+{
+    const Grid &g = r->g;
+    const int lnz = g.lnz, cur = r->cur;
+    T *uc = (T *)r->u[cur];
+    T *un = (T *)r->u[cur ^ 1];
+    auto timed = [&](int kind, auto fn) -> cudaError_t {
+        if (!prof) return fn();
+        cudaEvent_t a, b;
+        cudaEventCreate(&a);
+        cudaEventCreate(&b);
+        cudaEventRecord(a, s);
+        cudaError_t e = fn();
+        cudaEventRecord(b, s);
+        r->evs.push_back({kind, a, b});
+        return e;
+    };
+    auto vol = [&](int zl, int zh) {
+        return timed(0, [&] { return launch_volume<T>(g, uc, un, r->K, r->lambda, zl, zh, s, r->vplan, cur); });
+    };
+    auto bnd = [&](int64_t lo, int64_t hi) -> cudaError_t {
+        if (hi <= lo) return cudaSuccess;
+        return timed(1, [&] {
+            return launch_boundary<T>(r->MB, r->idx64, r->bpos, r->Kb, r->matb, lo, hi, r->nb, un, uc,
+                                      (T *)r->ub, (T *)r->gst, (T *)r->vst, (const T *)r->tab, r->M,
+                                      r->lambda, s);
+        });
+    };
+    const int zs = r->src_z >= 0 ? r->src_z - r->z0 : -1;
+    const bool src_edge = zs == 0 || zs == lnz - 1;
+    cudaError_t e = cudaSuccess;
+    if (phase == 0) {
+        e = vol(0, 1);
+        if (e == cudaSuccess && lnz > 1) e = vol(lnz - 1, lnz);
+        if (e == cudaSuccess) e = bnd(0, std::min(r->n_first_plane, r->nb));
+        if (e == cudaSuccess && lnz > 1) e = bnd(std::max(r->n_last_start, r->n_first_plane), r->nb);
+        if (e == cudaSuccess && src_edge) e = timed(2, [&] { return launch_src_rcv<T>(un, ctl_of<T>(r), s, 1); });
+    } else {
+        if (lnz > 2) e = vol(1, lnz - 1);
+        if (e == cudaSuccess && lnz > 2) e = bnd(r->n_first_plane, r->n_last_start);
+        if (e == cudaSuccess) e = timed(2, [&] { return launch_src_rcv<T>(un, ctl_of<T>(r), s, src_edge ? 2 : 3); });
+    }
+    return e;
+}
+
+static int kernels_per_phase(const rafd_room *r, int phase)
+{
+    const int lnz = r->g.lnz;
+    if (phase == 0) {
+        const int zs = r->src_z >= 0 ? r->src_z - r->z0 : -1;
+        return (lnz > 1 ? 2 : 1) + (r->n_first_plane > 0 ? 1 : 0) +
+               (lnz > 1 && r->nb > std::max(r->n_last_start, r->n_first_plane) ? 1 : 0) +
+               ((zs == 0 || zs == lnz - 1) ? 1 : 0);
+    }
+    return (lnz > 2 ? 1 : 0) + (lnz > 2 && r->n_last_start > r->n_first_plane ? 1 : 0) + 1;
+}
+
+// one NCCL-halo step of this rank
+template <typename T> static cudaError_t enqueue_step_nccl(rafd_room *r, bool prof)
+{
+    cudaError_t e = enqueue_phase<T>(r, 0, r->stream, prof);
+    if (e != cudaSuccess) return e;
+    if ((e = cudaEventRecord(r->ev_edge, r->stream)) != cudaSuccess) return e;
+    if ((e = cudaStreamWaitEvent(r->comm_stream, r->ev_edge, 0)) != cudaSuccess) return e;
+    e = halo_exchange(r->halo, r->u[r->cur ^ 1], (size_t)r->g.plane * sizeof(T), r->g.lnz, r->comm_stream);
+    if (e != cudaSuccess) return e;
+    if ((e = cudaEventRecord(r->ev_halo, r->comm_stream)) != cudaSuccess) return e;
+    e = enqueue_phase<T>(r, 1, r->stream, prof);
+    if (e != cudaSuccess) return e;
+    return cudaStreamWaitEvent(r->stream, r->ev_halo, 0);  // ghost planes ready for the next step
 }
 
 static int kernels_per_step(const rafd_room *r) { return 2 + (r->nb > 0 ? 1 : 0); }
@@ -652,10 +736,17 @@ template <typename T> static int step_t(rafd_room *r, int64_t nsteps)
         r->launches += (int64_t)kps * rafd_room::G;
     }
     for (; done < nsteps; done++) {
-        cudaError_t e = enqueue_step<T>(r, r->cur, r->stream, r->profiling);
-        if (e != cudaSuccess) return set_err(e == cudaErrorUnknown ? RAFD_E_NCCL : RAFD_E_CUDA, "step: %s", cudaGetErrorString(e));
+        cudaError_t e;
+        if (r->halo) {
+            e = enqueue_step_nccl<T>(r, r->profiling);
+            if (e == cudaErrorUnknown) return set_err(RAFD_E_NCCL, "%s", halo_last_error());
+            r->launches += kernels_per_phase(r, 0) + kernels_per_phase(r, 1);
+        } else {
+            e = enqueue_step<T>(r, r->cur, r->stream, r->profiling);
+            r->launches += kps;
+        }
+        if (e != cudaSuccess) return set_err(RAFD_E_CUDA, "step: %s", cudaGetErrorString(e));
         r->cur ^= 1;
-        r->launches += kps;
     }
     r->steps += nsteps;
     if (r->nrcv > 0) r->rec_count += nsteps;
@@ -683,36 +774,51 @@ template <typename T> static int step_group_t(rafd_room **rs, int n, int64_t nst
         if (rc) return rc;
     }
     for (int64_t st = 0; st < nsteps; st++) {
+        // phase 0 of every slab (after the neighbours finished copying out of
+        // the buffer this step overwrites... they read our u^{n}, which we
+        // overwrite one step later; waiting here is sufficient)
         for (int k = 0; k < n; k++) {
             rafd_room *r = rs[k];
             CK(cudaSetDevice(r->device));
-            if (st > 0) {  // neighbours must have finished reading our previous buffer
-                if (k > 0) CK(cudaStreamWaitEvent(r->stream, rs[k - 1]->ev_copied, 0));
-                if (k < n - 1) CK(cudaStreamWaitEvent(r->stream, rs[k + 1]->ev_copied, 0));
+            if (st > 0) {
+                if (k > 0) CK(cudaStreamWaitEvent(r->stream, rs[k - 1]->ev_halo, 0));
+                if (k < n - 1) CK(cudaStreamWaitEvent(r->stream, rs[k + 1]->ev_halo, 0));
             }
-            cudaError_t e = enqueue_step<T>(r, r->cur, r->stream, r->profiling);
+            cudaError_t e = enqueue_phase<T>(r, 0, r->stream, r->profiling);
             if (e != cudaSuccess) return set_err(RAFD_E_CUDA, "step: %s", cudaGetErrorString(e));
-            CK(cudaEventRecord(r->ev_done, r->stream));
-            r->launches += kernels_per_step(r);
+            CK(cudaEventRecord(r->ev_edge, r->stream));
+            r->launches += kernels_per_phase(r, 0);
         }
+        // halo: each slab pulls its ghost planes on its comm stream
         for (int k = 0; k < n; k++) {
             rafd_room *r = rs[k];
             CK(cudaSetDevice(r->device));
             const size_t pb = (size_t)r->g.plane * sizeof(T);
             char *mine = (char *)r->u[r->cur ^ 1];  // u^{n+1} of this slab
+            CK(cudaStreamWaitEvent(r->comm_stream, r->ev_edge, 0));
             if (k > 0) {
                 rafd_room *q = rs[k - 1];
-                CK(cudaStreamWaitEvent(r->stream, q->ev_done, 0));
+                CK(cudaStreamWaitEvent(r->comm_stream, q->ev_edge, 0));
                 const char *src = (const char *)q->u[q->cur ^ 1] + (size_t)q->g.lnz * pb;
-                CK(cudaMemcpyPeerAsync(mine, r->device, src, q->device, pb, r->stream));
+                CK(cudaMemcpyPeerAsync(mine, r->device, src, q->device, pb, r->comm_stream));
             }
             if (k < n - 1) {
                 rafd_room *q = rs[k + 1];
-                CK(cudaStreamWaitEvent(r->stream, q->ev_done, 0));
+                CK(cudaStreamWaitEvent(r->comm_stream, q->ev_edge, 0));
                 const char *src = (const char *)q->u[q->cur ^ 1] + pb;
-                CK(cudaMemcpyPeerAsync(mine + (size_t)(r->g.lnz + 1) * pb, r->device, src, q->device, pb, r->stream));
+                CK(cudaMemcpyPeerAsync(mine + (size_t)(r->g.lnz + 1) * pb, r->device, src, q->device, pb,
+                                       r->comm_stream));
             }
-            CK(cudaEventRecord(r->ev_copied, r->stream));
+            CK(cudaEventRecord(r->ev_halo, r->comm_stream));
+        }
+        // phase 1 (interior) overlapped with the copies
+        for (int k = 0; k < n; k++) {
+            rafd_room *r = rs[k];
+            CK(cudaSetDevice(r->device));
+            cudaError_t e = enqueue_phase<T>(r, 1, r->stream, r->profiling);
+            if (e != cudaSuccess) return set_err(RAFD_E_CUDA, "step: %s", cudaGetErrorString(e));
+            CK(cudaStreamWaitEvent(r->stream, r->ev_halo, 0));
+            r->launches += kernels_per_phase(r, 1);
         }
         for (int k = 0; k < n; k++) rs[k]->cur ^= 1;
     }

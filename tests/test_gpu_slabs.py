@@ -119,3 +119,29 @@ def test_c4_section_slabs_bitwise():
         s.read_field(out_curr=fs, out_prev=torch.empty_like(fs))
         assert torch.equal(fs, fw[a:b])
     assert float(fw.abs().max()) > 1e-4
+
+
+@pytest.mark.parametrize("where", ["first", "last", "interior"])
+def test_slab_source_and_receivers_on_edge_planes(where):
+    """Source / receivers on the planes handled by the edge phase (before the
+    halo exchange) and on interior planes; thin slabs (1 and 2 planes) too."""
+    dims = (30, 26, 12)
+    mask, mm, beta0, D, E, F = make_case("box", dims, 3, 8, seed=4)
+    plan = [(0, 1), (1, 3), (3, 7), (7, 12)]
+    z = {"first": 3, "last": 6, "interior": 5}[where]
+    src = (12, 11, z)
+    rcv = [(5, 5, 0), (7, 8, 1), (8, 9, 2), (9, 9, 3), (10, 10, 6), (11, 11, 7), (12, 12, 11), (3, 4, 5)]
+    whole = rafd.Room(mask, LAM, 32, beta0, D, E, F, matmap=mm)
+    slabs = [rafd.Room(mask, LAM, 32, beta0, D, E, F, matmap=mm, rank=k, nranks=4, z_begin=a, z_end=b)
+             for k, (a, b) in enumerate(plan)]
+    for r in [whole] + slabs:
+        r.set_source(src, I.gaussian_pulse(16, 2.0))
+        r.set_receivers(rcv)
+    whole.step(50)
+    rafd.rafd_step_group(slabs, 50)
+    cw = whole.read_field()[0]
+    cs = np.concatenate([s.read_field()[0] for s in slabs])
+    assert np.array_equal(cw, cs)
+    rw = whole.read_receivers()
+    rs = rafd.gather_receivers([s.read_receivers() for s in slabs], rcv, plan)
+    assert np.array_equal(rw, rs) and np.abs(rw).max() > 0
