@@ -105,6 +105,7 @@ typedef struct rafd_info {
     int32_t precision, n_materials, n_branches;
     int32_t z_begin, z_end;  /* planes owned                                           */
     int32_t pitch;           /* padded x pitch in elements                              */
+    int32_t fused;           /* 1: the boundary update runs inside the volume kernel     */
 } rafd_info;
 
 /* Per-kernel device times accumulated while profiling is on (CUDA events on

@@ -63,11 +63,26 @@ struct KernelTimes {
 
 // ------------------------------------------------------------------ launchers
 // (each returns cudaGetLastError() of its launch)
+// Arguments of the fused volume+boundary kernel (seg_first is set by the plan).
+template <typename T> struct FusedArgs {
+    const int32_t *seg_first;
+    const uint8_t *matb;
+    T *g, *v;
+    const T *tab;
+    int M, MB;
+    int64_t Nb;
+    T l;
+};
+
 // plan == nullptr selects the one-thread-per-voxel v0 kernel (A/B reference);
-// cur_idx = which of the two field buffers holds u^n (selects the TMA maps).
+// cur_idx = which of the two field buffers holds u^n (selects the TMA maps);
+// fa != nullptr (and a fused plan) applies the boundary update in the same pass.
 template <typename T>
 cudaError_t launch_volume(const Grid &g, const T *cur, T *nxt, const uint8_t *K, double lambda,
-                          int z_lo, int z_hi, cudaStream_t s, const void *plan, int cur_idx);
+                          int z_lo, int z_hi, cudaStream_t s, const void *plan, int cur_idx,
+                          const FusedArgs<T> *fa = nullptr);
+cudaError_t volume_plan_fuse(void *plan, const Grid &g, const uint8_t *K, int64_t Nb, cudaStream_t s);
+bool volume_plan_fused(const void *plan);
 template <typename T>
 cudaError_t volume_plan_create(const Grid &g, void *u0, void *u1, uint8_t *K, int nsm, void **plan);
 void volume_plan_destroy(void *plan);

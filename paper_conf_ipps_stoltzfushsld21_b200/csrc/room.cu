@@ -120,9 +120,24 @@ struct rafd_room {
     int src_z = -1;                                // global plane of the source (-1: none)
     // TMA tensor maps etc. of the volume kernel (nullptr => v0 kernel)
     void *vplan = nullptr;
+    bool fused = false;  // boundary update fused into the volume kernel
 };
 
 template <typename T> static Ctl<T> *ctl_of(rafd_room *r) { return (Ctl<T> *)r->ctl; }
+
+template <typename T> static FusedArgs<T> fused_args(const rafd_room *r)
+{
+    FusedArgs<T> f{};
+    f.matb = r->matb;
+    f.g = (T *)r->gst;
+    f.v = (T *)r->vst;
+    f.tab = (const T *)r->tab;
+    f.M = r->M;
+    f.MB = r->MB;
+    f.Nb = r->nb;
+    f.l = (T)r->lambda;
+    return f;
+}
 
 // every allocation carries 64 bytes of slack (vector loads / memsets of +16)
 static int dmalloc(rafd_room *r, void **p, size_t bytes)
@@ -355,6 +370,16 @@ template <typename T> static int create_t(rafd_room *r, const rafd_room_desc *d)
     CK(cudaMemcpy(r->ctl, &c, sizeof c, cudaMemcpyHostToDevice));
     const char *env = getenv("RAFD_VOLUME_KERNEL");
     if (!(env && strcmp(env, "v0") == 0)) CK(volume_plan_create<T>(g, r->u[0], r->u[1], r->K_alloc, r->nsm, &r->vplan));
+    // boundary update fused into the volume kernel with RAFD_FUSED=1 (DESIGN.md
+    // §6; needs the default tiling, MB <= 4, Nb < 2^31).  Off by default: the
+    // first fused form is latency-bound at x-wall rows (5.6 ms vs 2.55 ms).
+    const char *fz = getenv("RAFD_FUSED");
+    if (r->vplan && fz && strcmp(fz, "1") == 0 && r->MB <= 4 && nb < INT32_MAX) {
+        cudaError_t e = volume_plan_fuse(r->vplan, g, r->K, nb, r->stream);
+        if (e != cudaSuccess && e != cudaErrorNotSupported) CK(e);
+        cudaGetLastError();
+        r->fused = volume_plan_fused(r->vplan);
+    }
     return RAFD_OK;
 }
 
@@ -614,9 +639,12 @@ template <typename T> static cudaError_t enqueue_step(rafd_room *r, int cur, cud
         r->evs.push_back({kind, a, b});
         return e;
     };
-    cudaError_t e = timed(0, [&] { return launch_volume<T>(g, uc, un, r->K, r->lambda, 0, g.lnz, s, r->vplan, cur); });
+    const FusedArgs<T> fa = fused_args<T>(r);
+    cudaError_t e = timed(0, [&] {
+        return launch_volume<T>(g, uc, un, r->K, r->lambda, 0, g.lnz, s, r->vplan, cur, r->fused ? &fa : nullptr);
+    });
     if (e != cudaSuccess) return e;
-    if (r->nb > 0) {
+    if (r->nb > 0 && !r->fused) {
         e = timed(1, [&] {
             return launch_boundary<T>(r->MB, r->idx64, r->bpos, r->Kb, r->matb, 0, r->nb, r->nb, un, uc,
                                       (T *)r->ub, (T *)r->gst, (T *)r->vst, (const T *)r->tab, r->M,
@@ -650,11 +678,14 @@ template <typename T> static cudaError_t enqueue_phase(rafd_room *r, int phase, 
         r->evs.push_back({kind, a, b});
         return e;
     };
+    const FusedArgs<T> fa = fused_args<T>(r);
     auto vol = [&](int zl, int zh) {
-        return timed(0, [&] { return launch_volume<T>(g, uc, un, r->K, r->lambda, zl, zh, s, r->vplan, cur); });
+        return timed(0, [&] {
+            return launch_volume<T>(g, uc, un, r->K, r->lambda, zl, zh, s, r->vplan, cur, r->fused ? &fa : nullptr);
+        });
     };
     auto bnd = [&](int64_t lo, int64_t hi) -> cudaError_t {
-        if (hi <= lo) return cudaSuccess;
+        if (hi <= lo || r->fused) return cudaSuccess;
         return timed(1, [&] {
             return launch_boundary<T>(r->MB, r->idx64, r->bpos, r->Kb, r->matb, lo, hi, r->nb, un, uc,
                                       (T *)r->ub, (T *)r->gst, (T *)r->vst, (const T *)r->tab, r->M,
@@ -681,13 +712,14 @@ template <typename T> static cudaError_t enqueue_phase(rafd_room *r, int phase, 
 static int kernels_per_phase(const rafd_room *r, int phase)
 {
     const int lnz = r->g.lnz;
+    const int nbk = r->fused ? 0 : 1;  // boundary launches exist only in the two-kernel form
     if (phase == 0) {
         const int zs = r->src_z >= 0 ? r->src_z - r->z0 : -1;
-        return (lnz > 1 ? 2 : 1) + (r->n_first_plane > 0 ? 1 : 0) +
-               (lnz > 1 && r->nb > std::max(r->n_last_start, r->n_first_plane) ? 1 : 0) +
+        return (lnz > 1 ? 2 : 1) + nbk * (r->n_first_plane > 0 ? 1 : 0) +
+               nbk * (lnz > 1 && r->nb > std::max(r->n_last_start, r->n_first_plane) ? 1 : 0) +
                ((zs == 0 || zs == lnz - 1) ? 1 : 0);
     }
-    return (lnz > 2 ? 1 : 0) + (lnz > 2 && r->n_last_start > r->n_first_plane ? 1 : 0) + 1;
+    return (lnz > 2 ? 1 : 0) + nbk * (lnz > 2 && r->n_last_start > r->n_first_plane ? 1 : 0) + 1;
 }
 
 // one NCCL-halo step of this rank
@@ -705,7 +737,7 @@ template <typename T> static cudaError_t enqueue_step_nccl(rafd_room *r, bool pr
     return cudaStreamWaitEvent(r->stream, r->ev_halo, 0);  // ghost planes ready for the next step
 }
 
-static int kernels_per_step(const rafd_room *r) { return 2 + (r->nb > 0 ? 1 : 0); }
+static int kernels_per_step(const rafd_room *r) { return 2 + (r->nb > 0 && !r->fused ? 1 : 0); }
 
 template <typename T> static int build_graph(rafd_room *r, int parity)
 {
@@ -1046,6 +1078,7 @@ extern "C" int rafd_get_info(rafd_room *r, rafd_info *info)
     info->z_begin = r->z0;
     info->z_end = r->z1;
     info->pitch = (int32_t)r->g.pitch;
+    info->fused = r->fused ? 1 : 0;
     return RAFD_OK;
 }
 

@@ -58,7 +58,8 @@ class rafd_info(C.Structure):
                 ("bytes_per_step", C.c_int64), ("volume_bytes", C.c_int64),
                 ("boundary_bytes", C.c_int64), ("device_bytes", C.c_int64),
                 ("precision", C.c_int32), ("n_materials", C.c_int32), ("n_branches", C.c_int32),
-                ("z_begin", C.c_int32), ("z_end", C.c_int32), ("pitch", C.c_int32)]
+                ("z_begin", C.c_int32), ("z_end", C.c_int32), ("pitch", C.c_int32),
+                ("fused", C.c_int32)]
 
 
 class rafd_kernel_times(C.Structure):

@@ -15,6 +15,12 @@ pytestmark = pytest.mark.gpu
 LAM = 1.0 / math.sqrt(3.0)
 
 
+@pytest.fixture(autouse=True, params=["fused", "two-kernel"])
+def step_form(request, monkeypatch):
+    monkeypatch.setenv("RAFD_FUSED", "1" if request.param == "fused" else "0")
+    return request.param
+
+
 def make_case(shape, dims, MB, M, seed):
     nx, ny, nz = dims
     mask_t = I.make_mask(shape, nx, ny, nz, seed=seed)
