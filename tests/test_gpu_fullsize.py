@@ -57,3 +57,36 @@ def test_c4_full_size_two_steps_bitwise(orc):
     vo, go = o.read_branch_state()
     assert np.array_equal(vg, vo) and np.array_equal(gg, go)
     assert np.array_equal(g.read_receivers(), o.read_receivers())
+
+
+@pytest.mark.parametrize("name,precision,steps", [("C2a", 32, 30), ("C2b", 32, 30), ("C3", 32, 12), ("C3d", 64, 12)])
+def test_config_full_size_bitwise(orc, name, precision, steps):
+    """BASELINE.json configs[1..2] at full size (256^3 L-shape and dome with
+    FI-MM M=4; 512x384x256 box with FD-MM MB=3 M=8 in fp32 and fp64): a few
+    steps from a seeded random state plus the config's source, every voxel and
+    the receivers bitwise."""
+    cfg = I.CONFIGS[name]
+    nx, ny, nz = cfg["dims"]
+    mask_t = I.make_mask(cfg["shape"], nx, ny, nz)
+    mm = I.material_map(mask_t, cfg["rule"], cfg["M"]).numpy()
+    mask = mask_t.numpy()
+    beta0, D, E, F = I.config_materials(cfg)
+    g = rafd.Room(mask, LAM, precision, beta0, D, E, F, matmap=mm)
+    o = orc.OracleRoom(mask, LAM, precision, beta0, D, E, F, matmap=mm)
+    dt = np.float32 if precision == 32 else np.float64
+    rng = np.random.default_rng(7)
+    up = rng.uniform(-1, 1, mask.shape).astype(dt)
+    uc = rng.uniform(-1, 1, mask.shape).astype(dt)
+    src = I.source_position(cfg["dims"], mask)
+    rcv = I.receiver_positions(cfg["dims"], mask)
+    for r in (g, o):
+        r.set_state(up, uc)
+        r.set_source(src, I.impulse())
+        r.set_receivers(rcv)
+        r.step(steps)
+    assert np.array_equal(g.read_field()[0], o.read_field()[0])
+    assert np.array_equal(g.read_receivers(), o.read_receivers())
+    if cfg["MB"]:
+        vg, gg = g.read_branch_state()
+        vo, go = o.read_branch_state()
+        assert np.array_equal(vg, vo) and np.array_equal(gg, go)
