@@ -46,6 +46,10 @@ extern "C" {
 #define RAFD_E_NCCL -8       /* NCCL error or NCCL library not loadable                    */
 #define RAFD_E_STATE -9      /* call not valid in the current state                        */
 
+#define RAFD_SCHEME_TWO_KERNEL 0
+#define RAFD_SCHEME_LISTING1 1
+#define RAFD_SCHEME_NAIVE_FI 2
+
 #define RAFD_MAX_BRANCHES 8
 #define RAFD_MAX_MATERIALS 256
 
@@ -89,6 +93,16 @@ typedef struct rafd_room_desc {
      * A slab handle reads planes [z_begin-1, z_end] (clipped to the room), so a
      * rank may pass only those. */
     int32_t mask_z0;
+    /* Update scheme (readings R17 in DESIGN.md):
+     *  RAFD_SCHEME_TWO_KERNEL (0, default): Listings 2-4, any n_materials / n_branches;
+     *  RAFD_SCHEME_LISTING1  (1): the single kernel of Listing 1
+     *     with nbrs looked up and one admittance: n_materials = 1,
+     *     n_branches = 0, beta = beta0[0]; equal to scheme 0 up to rounding;
+     *  RAFD_SCHEME_NAIVE_FI  (2): Listing 6, the naive single
+     *     kernel: boundary points scale by the constants loss1, loss2
+     *     (next = loss1*((2-l2 K)u + l2 s - loss2*prev)); n_branches = 0, materials unused. */
+    int32_t scheme;
+    double loss1, loss2;
 } rafd_room_desc;
 
 typedef struct rafd_info {
@@ -106,6 +120,7 @@ typedef struct rafd_info {
     int32_t z_begin, z_end;  /* planes owned                                           */
     int32_t pitch;           /* padded x pitch in elements                              */
     int32_t fused;           /* 1: the boundary update runs inside the volume kernel     */
+    int32_t scheme;          /* RAFD_SCHEME_*                                          */
 } rafd_info;
 
 /* Per-kernel device times accumulated while profiling is on (CUDA events on

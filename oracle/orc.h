@@ -86,6 +86,10 @@ int  orc_set_receivers(orc_room *r, int32_t n, const int32_t *xyz);
  * outside voxels are forced to +0.  v, g: T-typed [MB][Nb] (NULL => keep). */
 int  orc_set_state(orc_room *r, const void *u_prev, const void *u_curr, const void *v, const void *g);
 int  orc_step(orc_room *r, int64_t nsteps);
+/* Single-kernel schemes of the paper: 0 = Listings 2-4 (default),
+ * 1 = Listing 1 (n_materials = 1, MB = 0, beta = beta0[0]),
+ * 2 = Listing 6 naive FI (constants loss1, loss2, reading R17). */
+int  orc_set_scheme(orc_room *r, int32_t scheme, double loss1, double loss2);
 int  orc_read_receivers(orc_room *r, double *out, int64_t cap, int64_t *n_written);
 /* Fields as T-typed [nz][ny][nx]: u^n (curr) and u^{n-1} (prev).  NULL => skip. */
 int  orc_read_field(orc_room *r, void *u_curr, void *u_prev);

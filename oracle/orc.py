@@ -62,6 +62,7 @@ def lib():
         L.orc_set_receivers.argtypes = [P, C.c_int32, P]
         L.orc_set_state.argtypes = [P, P, P, P, P]
         L.orc_step.argtypes = [P, C.c_int64]
+        L.orc_set_scheme.argtypes = [P, C.c_int32, C.c_double, C.c_double]
         L.orc_read_receivers.argtypes = [P, P, C.c_int64, C.POINTER(C.c_int64)]
         L.orc_read_field.argtypes = [P, P, P]
         L.orc_read_branch_state.argtypes = [P, P, P]
@@ -162,6 +163,9 @@ class OracleRoom:
 
     def step(self, n):
         _check(lib().orc_step(self.h, int(n)))
+
+    def set_scheme(self, scheme, loss1=1.0, loss2=1.0):
+        _check(lib().orc_set_scheme(self.h, int(scheme), float(loss1), float(loss2)))
 
     def read_receivers(self, cap=None):
         if self.nrcv == 0:

@@ -72,9 +72,13 @@ template <typename T> struct FusedArgs {
     int M, MB;
     int64_t Nb;
     T l;
+    int scheme;      // 0: Listing 2 volume; 1: Listing 1 single kernel; 2: Listing 6 naive FI
+    T beta1;         // Listing 1 admittance
+    T loss1, loss2;  // Listing 6 constants
 };
 
 // plan == nullptr selects the one-thread-per-voxel v0 kernel (A/B reference);
+// fa->scheme != 0 selects a single-kernel scheme (then no boundary kernel runs);
 // cur_idx = which of the two field buffers holds u^n (selects the TMA maps);
 // fa != nullptr (and a fused plan) applies the boundary update in the same pass.
 template <typename T>

@@ -121,6 +121,8 @@ struct rafd_room {
     // TMA tensor maps etc. of the volume kernel (nullptr => v0 kernel)
     void *vplan = nullptr;
     bool fused = false;  // boundary update fused into the volume kernel
+    int scheme = 0;      // RAFD_SCHEME_*
+    double beta1 = 0, loss1 = 1, loss2 = 1;
 };
 
 template <typename T> static Ctl<T> *ctl_of(rafd_room *r) { return (Ctl<T> *)r->ctl; }
@@ -136,6 +138,10 @@ template <typename T> static FusedArgs<T> fused_args(const rafd_room *r)
     f.MB = r->MB;
     f.Nb = r->nb;
     f.l = (T)r->lambda;
+    f.scheme = r->scheme;
+    f.beta1 = (T)r->beta1;
+    f.loss1 = (T)r->loss1;
+    f.loss2 = (T)r->loss2;
     return f;
 }
 
@@ -179,6 +185,11 @@ static int validate(const rafd_room_desc *d)
                 return set_err(RAFD_E_NONPASSIVE, "D, E, F of material %d branch %d must be finite and >= 0", i, b);
         }
     }
+    if (d->scheme < 0 || d->scheme > 2) return set_err(RAFD_E_INVAL, "scheme must be 0, 1 or 2");
+    if (d->scheme == 1 && (m->n_materials != 1 || m->n_branches != 0))
+        return set_err(RAFD_E_INVAL, "Listing 1 has one admittance: n_materials = 1 and n_branches = 0");
+    if (d->scheme == 2 && (m->n_branches != 0 || !std::isfinite(d->loss1) || !std::isfinite(d->loss2)))
+        return set_err(RAFD_E_INVAL, "Listing 6 needs n_branches = 0 and finite loss1, loss2");
     if (d->mask_z0 < 0 || d->mask_z0 > std::max(0, (d->nranks > 1 ? d->z_begin : 0) - 1))
         return set_err(RAFD_E_INVAL, "mask_z0 must be <= the first plane read (z_begin-1, clipped)");
     if (d->nranks > 1) {
@@ -374,7 +385,7 @@ template <typename T> static int create_t(rafd_room *r, const rafd_room_desc *d)
     // §6; needs the default tiling, MB <= 4, Nb < 2^31).  Off by default: the
     // first fused form is latency-bound at x-wall rows (5.6 ms vs 2.55 ms).
     const char *fz = getenv("RAFD_FUSED");
-    if (r->vplan && fz && strcmp(fz, "1") == 0 && r->MB <= 4 && nb < INT32_MAX) {
+    if (r->vplan && fz && strcmp(fz, "1") == 0 && r->MB <= 4 && nb < INT32_MAX && r->scheme == 0) {
         cudaError_t e = volume_plan_fuse(r->vplan, g, r->K, nb, r->stream);
         if (e != cudaSuccess && e != cudaErrorNotSupported) CK(e);
         cudaGetLastError();
@@ -406,6 +417,10 @@ extern "C" int rafd_create(const rafd_room_desc *d, rafd_room **out)
     r->ny = d->ny;
     r->nz = d->nz;
     r->lambda = d->lambda;
+    r->scheme = d->scheme;
+    r->beta1 = d->mat->beta0[0];
+    r->loss1 = d->loss1;
+    r->loss2 = d->loss2;
     r->rank = d->nranks > 1 ? d->rank : 0;
     r->nranks = d->nranks > 1 ? d->nranks : 1;
     r->z0 = r->nranks > 1 ? d->z_begin : 0;
@@ -641,10 +656,11 @@ template <typename T> static cudaError_t enqueue_step(rafd_room *r, int cur, cud
     };
     const FusedArgs<T> fa = fused_args<T>(r);
     cudaError_t e = timed(0, [&] {
-        return launch_volume<T>(g, uc, un, r->K, r->lambda, 0, g.lnz, s, r->vplan, cur, r->fused ? &fa : nullptr);
+        return launch_volume<T>(g, uc, un, r->K, r->lambda, 0, g.lnz, s, r->vplan, cur,
+                                (r->fused || r->scheme) ? &fa : nullptr);
     });
     if (e != cudaSuccess) return e;
-    if (r->nb > 0 && !r->fused) {
+    if (r->nb > 0 && !r->fused && !r->scheme) {
         e = timed(1, [&] {
             return launch_boundary<T>(r->MB, r->idx64, r->bpos, r->Kb, r->matb, 0, r->nb, r->nb, un, uc,
                                       (T *)r->ub, (T *)r->gst, (T *)r->vst, (const T *)r->tab, r->M,
@@ -681,11 +697,12 @@ template <typename T> static cudaError_t enqueue_phase(rafd_room *r, int phase, 
     const FusedArgs<T> fa = fused_args<T>(r);
     auto vol = [&](int zl, int zh) {
         return timed(0, [&] {
-            return launch_volume<T>(g, uc, un, r->K, r->lambda, zl, zh, s, r->vplan, cur, r->fused ? &fa : nullptr);
+            return launch_volume<T>(g, uc, un, r->K, r->lambda, zl, zh, s, r->vplan, cur,
+                                    (r->fused || r->scheme) ? &fa : nullptr);
         });
     };
     auto bnd = [&](int64_t lo, int64_t hi) -> cudaError_t {
-        if (hi <= lo || r->fused) return cudaSuccess;
+        if (hi <= lo || r->fused || r->scheme) return cudaSuccess;
         return timed(1, [&] {
             return launch_boundary<T>(r->MB, r->idx64, r->bpos, r->Kb, r->matb, lo, hi, r->nb, un, uc,
                                       (T *)r->ub, (T *)r->gst, (T *)r->vst, (const T *)r->tab, r->M,
@@ -712,7 +729,7 @@ template <typename T> static cudaError_t enqueue_phase(rafd_room *r, int phase, 
 static int kernels_per_phase(const rafd_room *r, int phase)
 {
     const int lnz = r->g.lnz;
-    const int nbk = r->fused ? 0 : 1;  // boundary launches exist only in the two-kernel form
+    const int nbk = (r->fused || r->scheme) ? 0 : 1;  // boundary launches exist only in the two-kernel form
     if (phase == 0) {
         const int zs = r->src_z >= 0 ? r->src_z - r->z0 : -1;
         return (lnz > 1 ? 2 : 1) + nbk * (r->n_first_plane > 0 ? 1 : 0) +
@@ -737,7 +754,7 @@ template <typename T> static cudaError_t enqueue_step_nccl(rafd_room *r, bool pr
     return cudaStreamWaitEvent(r->stream, r->ev_halo, 0);  // ghost planes ready for the next step
 }
 
-static int kernels_per_step(const rafd_room *r) { return 2 + (r->nb > 0 && !r->fused ? 1 : 0); }
+static int kernels_per_step(const rafd_room *r) { return 2 + (r->nb > 0 && !r->fused && !r->scheme ? 1 : 0); }
 
 template <typename T> static int build_graph(rafd_room *r, int parity)
 {
@@ -1079,6 +1096,7 @@ extern "C" int rafd_get_info(rafd_room *r, rafd_info *info)
     info->z_end = r->z1;
     info->pitch = (int32_t)r->g.pitch;
     info->fused = r->fused ? 1 : 0;
+    info->scheme = r->scheme;
     return RAFD_OK;
 }
 

@@ -26,6 +26,9 @@ RAFD_E_NOMEM = -6
 RAFD_E_CUDA = -7
 RAFD_E_NCCL = -8
 RAFD_E_STATE = -9
+RAFD_SCHEME_TWO_KERNEL = 0
+RAFD_SCHEME_LISTING1 = 1
+RAFD_SCHEME_NAIVE_FI = 2
 
 # every symbol include/rafd.h declares (checked by tests/test_abi.py)
 ABI_SYMBOLS = [
@@ -49,7 +52,8 @@ class rafd_room_desc(C.Structure):
                 ("mat", C.POINTER(rafd_materials)), ("device", C.c_int32),
                 ("cuda_stream", C.c_void_p), ("rank", C.c_int32), ("nranks", C.c_int32),
                 ("nccl_id", C.c_void_p), ("z_begin", C.c_int32), ("z_end", C.c_int32),
-                ("mask_z0", C.c_int32)]
+                ("mask_z0", C.c_int32), ("scheme", C.c_int32), ("loss1", C.c_double),
+                ("loss2", C.c_double)]
 
 
 class rafd_info(C.Structure):
@@ -59,7 +63,7 @@ class rafd_info(C.Structure):
                 ("boundary_bytes", C.c_int64), ("device_bytes", C.c_int64),
                 ("precision", C.c_int32), ("n_materials", C.c_int32), ("n_branches", C.c_int32),
                 ("z_begin", C.c_int32), ("z_end", C.c_int32), ("pitch", C.c_int32),
-                ("fused", C.c_int32)]
+                ("fused", C.c_int32), ("scheme", C.c_int32)]
 
 
 class rafd_kernel_times(C.Structure):
@@ -142,7 +146,7 @@ class Room:
 
     def __init__(self, mask, lam, precision, beta0, D=None, E=None, F=None, matmap=None,
                  device=0, stream=None, rank=0, nranks=1, nccl_id=None, z_begin=0, z_end=0,
-                 mask_z0=0, dims=None):
+                 mask_z0=0, dims=None, scheme=0, loss1=1.0, loss2=1.0):
         L = lib()
         # dims = (nx, ny, nz) of the room when `mask` holds only planes [mask_z0, ...)
         nz, ny, nx = (int(s) for s in mask.shape)
@@ -174,7 +178,7 @@ class Room:
         d = rafd_room_desc(nx, ny, nz, _addr(mask), _addr(matmap), float(lam), int(precision),
                            C.pointer(self._mat), int(device), stream, int(rank), int(nranks),
                            None if idbuf is None else C.addressof(idbuf), int(z_begin), int(z_end),
-                           int(mask_z0))
+                           int(mask_z0), int(scheme), float(loss1), float(loss2))
         h = C.c_void_p()
         _check(L.rafd_create(C.byref(d), C.byref(h)))
         self.h = h

@@ -253,3 +253,40 @@ def test_volume_tile_configs_bitwise(orc, cfg, precision, monkeypatch):
         g0.set_source(src, I.gaussian_pulse(30, 4.0))
         g0.step(60)
         assert_close(o.read_field()[0], g0.read_field()[0], precision, "v0")
+
+
+@pytest.mark.parametrize("scheme", [1, 2])
+@pytest.mark.parametrize("precision", [32, 64])
+@pytest.mark.parametrize("kernel", ["tma", "v0"])
+def test_single_kernel_schemes_bitwise(orc, scheme, precision, kernel, monkeypatch):
+    """Listing 1 (one admittance) and Listing 6 (naive FI,
+    constants loss1/loss2) as single kernels, vs the oracle's schemes."""
+    if kernel == "v0":
+        monkeypatch.setenv("RAFD_VOLUME_KERNEL", "v0")
+    mask = I.dome_mask(150, 70, 40).numpy()
+    beta = [0.27]
+    c = 0.12
+    kw = dict(scheme=scheme, loss1=1.0 / (1.0 + c), loss2=1.0 - c)
+    o = orc.OracleRoom(mask, LAM, precision, beta)
+    o.set_scheme(scheme, kw["loss1"], kw["loss2"])
+    g = rafd.Room(mask, LAM, precision, beta, **kw)
+    assert g.get_info()["scheme"] == scheme and g.get_info()["fused"] == 0
+    src = I.snap_inside(mask, (70, 30, 20))
+    rcv = [I.snap_inside(mask, p) for p in [(10, 30, 5), (75, 35, 20), (140, 40, 30)]]
+    for r in (o, g):
+        r.set_source(src, I.gaussian_pulse(30, 4.0))
+        r.set_receivers(rcv)
+        r.step(120)
+    assert_close(o.read_field()[0], g.read_field()[0], precision, f"scheme {scheme}")
+    assert_close(o.read_receivers(), g.read_receivers(), precision, "receivers")
+    assert g.launch_count() == 2 * 120          # one volume kernel + source/receivers per step
+
+
+def test_scheme_validation():
+    mask = np.ones((6, 6, 6), np.uint8)
+    with pytest.raises(rafd.RafdError) as e:
+        rafd.Room(mask, LAM, 32, [0.1, 0.2], scheme=1)
+    assert e.value.code == rafd.RAFD_E_INVAL
+    with pytest.raises(rafd.RafdError) as e:
+        rafd.Room(mask, LAM, 32, [0.0], D=[[1.0]], E=[[1.0]], F=[[1.0]], scheme=2)
+    assert e.value.code == rafd.RAFD_E_INVAL

@@ -574,3 +574,72 @@ def test_fp32_is_single_precision_and_close_to_fp64(orc):
         out[p] = r.read_receivers()[0]
     d = np.abs(out[32] - out[64]).max() / np.abs(out[64]).max()
     assert 0 < d < 1e-2            # fp32 vs fp64 differ by 3e-4..7e-3 of peak
+
+
+# ---------------------------------------------------------------- single-kernel schemes (f3)
+
+
+def test_listing1_equals_two_kernel_fi(orc):
+    """Listing 1 (one kernel) and Listings 2+3 (two kernels)
+    are the same update written two ways: equal to rounding for beta > 0
+    (1e-12 of peak after 300 fp64 steps), and bitwise for beta = 0 (the
+    boundary branch degenerates to t - prev exactly)."""
+    mask = I.blob_mask(12, 11, 9, seed=31, fill=0.85).numpy()
+    up, uc = _rand_state(mask, 12, np.float64)
+    for beta, bitwise in ((0.3, False), (0.0, True)):
+        a = orc.OracleRoom(mask, LAM, 64, [beta])
+        b = orc.OracleRoom(mask, LAM, 64, [beta])
+        b.set_scheme(1)
+        for r in (a, b):
+            r.set_state(up, uc)
+            r.step(300)
+        fa, fb = a.read_field()[0], b.read_field()[0]
+        if bitwise:
+            assert np.array_equal(fa, fb)
+        else:
+            assert not np.array_equal(fa, fb)            # really a different rounding sequence
+            assert np.abs(fa - fb).max() <= 1e-12 * np.abs(fa).max()
+    with pytest.raises(orc.OracleError):
+        orc.OracleRoom(mask, LAM, 64, [0.1, 0.2]).set_scheme(1)   # one admittance only
+
+
+def test_listing1_energy_decays(orc):
+    mask = I.ellipsoid_mask(14, 12, 10).numpy()
+    up, uc = _rand_state(mask, 13, np.float64)
+    r = orc.OracleRoom(mask, LAM, 64, [0.2])
+    r.set_scheme(1)
+    r.set_state(up, uc)
+    h = _energy_series(r, 200)
+    assert np.all(np.diff(h) <= 1e-13 * h[0]) and h[-1] < 0.9 * h[0]
+
+
+def test_listing6_naive_rigid_is_dct_mode(orc):
+    """Listing 6 with loss1 = loss2 = 1 is the rigid
+    leapfrog summed in LIFT's neighbour order: the DCT-II modes are exact."""
+    dims = (12, 10, 8)
+    nx, ny, nz = dims
+    for m in [(2, 1, 3), (11, 9, 7)]:
+        phi = dct_mode(dims, m)
+        w = mode_theta(dims, m, LAM)
+        r = orc.OracleRoom(np.ones((nz, ny, nx), np.uint8), LAM, 64, [0.0])
+        r.set_scheme(2, 1.0, 1.0)
+        r.set_state(u_prev=math.cos(w) * phi, u_curr=phi)
+        r.step(1000)
+        assert np.abs(r.read_field()[0] - math.cos(1000 * w) * phi).max() < 1e-11
+
+
+def test_listing6_naive_energy(orc):
+    """With loss1 = 1/(1+c), loss2 = 1-c the naive update is
+    u+ - 2u + u- = l^2 sum(u_j - u) - c (u+ - u-) at boundary points: H is
+    non-increasing for c > 0 and conserved for c = 0."""
+    mask = I.ellipsoid_mask(14, 12, 10).numpy()
+    up, uc = _rand_state(mask, 14, np.float64)
+    for c in (0.0, 0.15):
+        r = orc.OracleRoom(mask, LAM, 64, [0.0])
+        r.set_scheme(2, 1.0 / (1.0 + c), 1.0 - c)
+        r.set_state(up, uc)
+        h = _energy_series(r, 200)
+        if c == 0.0:
+            assert np.abs(h / h[0] - 1).max() < 1e-12
+        else:
+            assert np.all(np.diff(h) <= 1e-13 * h[0]) and h[-1] < 0.95 * h[0]

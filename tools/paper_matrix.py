@@ -91,6 +91,33 @@ def main():
                     r.destroy()
                     del r
                     torch.cuda.empty_cache()
+            # Table IV's kernel itself: the naive one-kernel FI of Listing 6 (scheme 2), box only
+            if shape == "box":
+                for prec in (32, 64):
+                    c = 0.1
+                    r = rafd.Room(mask, LAM, prec, [0.0], scheme=2, loss1=1 / (1 + c), loss2=1 - c)
+                    nin = r.get_info()["n_inside"]
+                    r.set_source(I.source_position((nx, ny, nz)), I.impulse())
+                    r.step(a.warmup)
+                    r.synchronize()
+                    r.set_profiling(True)
+                    r.step(a.steps)
+                    kt = r.get_kernel_times()
+                    r.set_profiling(False)
+                    vol = kt["volume_ms"] / kt["volume_launches"]
+                    pv = paper_best(tables, "table_iv_fi_naive_one_kernel", int(size), "box", prec)
+                    row = {"room": f"{nx}x{ny}x{nz}", "shape": shape, "boundary": "naive FI (Listing 6, 1 kernel)",
+                           "precision": prec, "n_inside": nin, "n_boundary": r.get_info()["n_boundary"],
+                           "volume_ms": round(vol, 4), "boundary_ms": 0.0, "step_ms": round(vol, 4),
+                           "step_gvox_s": round(nin / (vol * 1e-3) / 1e9, 2), "volume_gvox_s": round(nin / (vol * 1e-3) / 1e9, 2),
+                           "boundary_gpts_s": None, "step_algorithmic_gbs": round(nin * (1 + 3 * prec // 8) / (vol * 1e-3) / 1e9, 1),
+                           "paper_boundary_best": None, "paper_fi_one_kernel_best": pv,
+                           "kernel_speedup_vs_paper_table_iv": round(pv["ms"] / vol, 1)}
+                    out.append(row)
+                    print(json.dumps(row), flush=True)
+                    r.destroy()
+                    del r
+                    torch.cuda.empty_cache()
             del mask, mm
     os.makedirs(os.path.join(ROOT, "profiles"), exist_ok=True)
     json.dump(out, open(os.path.join(ROOT, "profiles", f"{a.tag}_paper_matrix.json"), "w"), indent=1)
@@ -101,7 +128,8 @@ def main():
         pb = r["paper_boundary_best"]
         pv = r["paper_fi_one_kernel_best"]
         lines.append(f"| {r['room']} | {r['shape']} | {r['boundary']} | fp{r['precision']} | {r['n_boundary']} | "
-                     f"{r['volume_ms']} | {r['boundary_ms']} ({r['boundary_gpts_s']}) | {r['step_ms']} ({r['step_gvox_s']}) | "
+                     f"{r['volume_ms']} | " + (f"{r['boundary_ms']} ({r['boundary_gpts_s']})" if r['boundary_gpts_s'] else "—") +
+                     f" | {r['step_ms']} ({r['step_gvox_s']}) | "
                      + (f"{pb['ms']} ({pb['gpu']}, {pb['line']})" if pb else "—") + " | "
                      + (f"{pv['ms']} ({pv['gpu']}, {pv['line']})" if pv else "—") + " |")
     open(os.path.join(ROOT, "profiles", f"{a.tag}_paper_matrix.md"), "w").write(
