@@ -150,12 +150,38 @@ def slab_plan_box(nx, ny, nz, precision, MB, nranks):
     return list(zip(cuts[:-1], cuts[1:]))
 
 
+def _reduce(t, op):
+    """all_reduce a float64 tensor on the process group's device (NCCL: CUDA, gloo: CPU)."""
+    if torch.distributed.get_backend() == "nccl":
+        t = t.cuda()
+    else:
+        t = t.cpu()
+    torch.distributed.all_reduce(t, op=op)
+    return t.cpu()
+
+
+def bench_device(local_rank):
+    """GPU of this rank; RAFD_BENCH_DEVICE pins every rank to one GPU (a
+    multi-rank run on a single GPU, IPC transport, for testing)."""
+    d = os.environ.get("RAFD_BENCH_DEVICE")
+    return int(d) if d is not None else local_rank
+
+
+def connect_ipc(room, rank, world):
+    """Exchange the slabs' CUDA-IPC blobs and connect neighbours (transport 'ipc')."""
+    blobs = [None] * world
+    torch.distributed.all_gather_object(blobs, room.ipc_handle())
+    room.ipc_connect(blobs[rank - 1] if rank > 0 else None, blobs[rank + 1] if rank < world - 1 else None)
+    torch.distributed.barrier()
+
+
 def run_rafd(args, rank, world, local_rank):
     from paper_conf_ipps_stoltzfushsld21_b200 import build, rafd
     if rank == 0:
         build.build()
     if world > 1:
         torch.distributed.barrier()
+    local_rank = bench_device(local_rank)
     dev = torch.device("cuda", local_rank)
     torch.cuda.set_device(dev)
     cfg = workload(args.config, world)
@@ -165,7 +191,7 @@ def run_rafd(args, rank, world, local_rank):
     plan = slab_plan_box(nx, ny, nz, prec, cfg["MB"], world)
     z0, z1 = plan[rank]
     nccl_id = None
-    if world > 1:
+    if world > 1 and args.transport == "nccl":
         obj = [rafd.rafd_nccl_unique_id() if rank == 0 else None]
         torch.distributed.broadcast_object_list(obj, src=0)
         nccl_id = obj[0]
@@ -175,6 +201,8 @@ def run_rafd(args, rank, world, local_rank):
     room = rafd.Room(mask, LAM, prec, beta0, D, E, F, matmap=mm, device=local_rank,
                      stream=stream.cuda_stream, rank=rank, nranks=world, nccl_id=nccl_id,
                      z_begin=z0, z_end=z1, mask_z0=mz0, dims=(nx, ny, nz))
+    if world > 1 and args.transport == "ipc":
+        connect_ipc(room, rank, world)
     t_create = time.perf_counter() - t_c
     del mask, mm
     torch.cuda.empty_cache()
@@ -213,10 +241,8 @@ def run_rafd(args, rank, world, local_rank):
                       kt["volume_ms"], kt["boundary_ms"], kt["other_ms"]], dtype=torch.float64,
                      device=dev)
     if world > 1:
-        mx = t.clone()
-        torch.distributed.all_reduce(mx, op=torch.distributed.ReduceOp.MAX)
-        sm = t.clone()
-        torch.distributed.all_reduce(sm, op=torch.distributed.ReduceOp.SUM)
+        mx = _reduce(t.clone(), torch.distributed.ReduceOp.MAX)
+        sm = _reduce(t.clone(), torch.distributed.ReduceOp.SUM)
     else:
         mx = sm = t
     ms_max = float(mx[0])
@@ -228,8 +254,10 @@ def run_rafd(args, rank, world, local_rank):
     if rank == 0:
         peak, peak_src = peaks()
         fused = bool(info["fused"])
-        vol_ms = kt["volume_ms"] / max(1, kt["volume_launches"])
-        bnd_ms = kt["boundary_ms"] / max(1, kt["boundary_launches"]) if kt["boundary_launches"] else 0.0
+        # per step: one volume launch per step on one GPU; a slab splits it into
+        # edge-plane and interior launches, so sum them per step
+        vol_ms = kt["volume_ms"] / args.steps
+        bnd_ms = kt["boundary_ms"] / args.steps if kt["boundary_launches"] else 0.0
         # the fused kernel moves the whole step's algorithmic bytes (volume + boundary)
         vol_bytes = info["bytes_per_step"] if fused else info["volume_bytes"]
         vol_gbs = vol_bytes / (vol_ms * 1e-3) / 1e9
@@ -254,6 +282,7 @@ def run_rafd(args, rank, world, local_rank):
                 "workload": f"{args.config}: {nx}x{ny}x{nz} box hall, FD-MM MB={cfg['MB']} M={cfg['M']}, "
                             f"fp{prec}" + (f", {world} z-slabs" if world > 1 else ""),
                 "room_dims_xyz": [nx, ny, nz], "n_inside": int(n_in_total),
+                "halo_transport": args.transport if world > 1 else None,
                 "n_boundary_rank0": info["n_boundary"], "parallelism": f"z-slab x{world}",
                 "l2": "inputs larger than L2 (working set %.1f GB/GPU vs 126 MB L2)" % (info["device_bytes"] / 1e9),
                 "timed": "profiled launches (CUDA events around every kernel) on the room stream",
@@ -263,11 +292,12 @@ def run_rafd(args, rank, world, local_rank):
                 "achieved": round(vol_gbs, 1), "peak": peak,
                 "unit": "GB/s", "frac": round(vol_gbs / peak, 4), "traffic": traffic,
                 "algorithmic_bytes_per_launch": vol_bytes,
-                "avg_launch_ms": round(vol_ms, 5), "peak_source": peak_src,
+                "avg_launch_ms": round(vol_ms, 5), "launches_per_step": kt["volume_launches"] // args.steps,
+                "peak_source": peak_src,
             },
             "kernels": {
                 "volume_ms_per_step": round(vol_ms, 5), "boundary_ms_per_step": round(bnd_ms, 5),
-                "other_ms_per_step": round(kt["other_ms"] / max(1, kt["other_launches"]), 5),
+                "other_ms_per_step": round(kt["other_ms"] / args.steps, 5),
                 "boundary_gbs": None if bnd_gbs is None else round(bnd_gbs, 1),
                 "boundary_share": round(bnd_ms / (ms_max / args.steps), 4),
                 "fused_boundary": fused,
@@ -283,7 +313,8 @@ def run_rafd(args, rank, world, local_rank):
     del room
     torch.cuda.synchronize()
     torch.cuda.empty_cache()
-    e2e = run_e2e(args, cfg, prec, beta0, D, E, F, rank, world, local_rank, plan, nccl_id is not None)
+    e2e = run_e2e(args, cfg, prec, beta0, D, E, F, rank, world, local_rank, plan,
+                  world > 1 and args.transport == "nccl")
     if rank == 0:
         out["e2e"] = e2e
     return out
@@ -297,6 +328,7 @@ def run_e2e(args, cfg, prec, beta0, D, E, F, rank, world, local_rank, plan, mult
     from paper_conf_ipps_stoltzfushsld21_b200 import rafd
     nx, ny, nz = cfg["room"]
     z0, z1 = plan[rank]
+    local_rank = bench_device(local_rank)
     mask_d, mm_d, mz0 = slab_inputs(cfg, z0, z1, torch.device("cuda", local_rank))
     mask_h = torch.empty(mask_d.shape, dtype=torch.uint8, pin_memory=True)
     mm_h = torch.empty(mm_d.shape, dtype=torch.uint8, pin_memory=True)
@@ -309,6 +341,7 @@ def run_e2e(args, cfg, prec, beta0, D, E, F, rank, world, local_rank, plan, mult
         obj = [rafd.rafd_nccl_unique_id() if rank == 0 else None]
         torch.distributed.broadcast_object_list(obj, src=0)
         nccl_id = obj[0]
+    ipc = world > 1 and args.transport == "ipc"
     sig = I.impulse()
     rcv = I.receiver_positions((nx, ny, nz))
     steps = args.steps
@@ -319,6 +352,8 @@ def run_e2e(args, cfg, prec, beta0, D, E, F, rank, world, local_rank, plan, mult
     room = rafd.Room(mask_h.numpy(), LAM, prec, beta0, D, E, F, matmap=mm_h.numpy(), device=local_rank,
                      rank=rank, nranks=world, nccl_id=nccl_id, z_begin=z0, z_end=z1, mask_z0=mz0,
                      dims=(nx, ny, nz))
+    if ipc:
+        connect_ipc(room, rank, world)
     room.set_source(I.source_position((nx, ny, nz)), sig)
     room.set_receivers(rcv)
     d2h = 0
@@ -332,10 +367,8 @@ def run_e2e(args, cfg, prec, beta0, D, E, F, rank, world, local_rank, plan, mult
     room.destroy()
     el = torch.tensor([t1 - t0, float(n_in)], dtype=torch.float64, device=torch.device("cuda", local_rank))
     if world > 1:
-        mx = el.clone()
-        torch.distributed.all_reduce(mx, op=torch.distributed.ReduceOp.MAX)
-        sm = el.clone()
-        torch.distributed.all_reduce(sm, op=torch.distributed.ReduceOp.SUM)
+        mx = _reduce(el.clone(), torch.distributed.ReduceOp.MAX)
+        sm = _reduce(el.clone(), torch.distributed.ReduceOp.SUM)
         tmax, n_tot = float(mx[0]), float(sm[1])
     else:
         tmax, n_tot = float(el[0]), float(el[1])
@@ -409,6 +442,9 @@ def main():
     ap.add_argument("--config", default="C4")
     ap.add_argument("--precision", type=int, default=None)
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--transport", default="nccl", choices=["nccl", "ipc"],
+                    help="halo exchange for --gpus > 1: NCCL send/recv, or CUDA-IPC peer copies "
+                         "ordered by GPU-side stream waits (rafd_ipc_connect)")
     args = ap.parse_args()
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
@@ -418,8 +454,12 @@ def main():
             print(json.dumps(run_reference(args)), flush=True)
         return
     if world > 1:
-        torch.cuda.set_device(local_rank)
-        torch.distributed.init_process_group("nccl", device_id=torch.device("cuda", local_rank))
+        dev = bench_device(local_rank)
+        torch.cuda.set_device(dev)
+        if args.transport == "nccl":
+            torch.distributed.init_process_group("nccl", device_id=torch.device("cuda", dev))
+        else:  # IPC halo: the process group only carries the blobs and the timing reductions
+            torch.distributed.init_process_group("gloo")
     out = run_rafd(args, rank, world, local_rank)
     if rank == 0:
         if world == 1 and not args.no_cpu_baseline:

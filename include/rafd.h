@@ -170,6 +170,20 @@ int rafd_step(rafd_room *r, int64_t nsteps);
  * a group.  rafd_step on a slab without nccl_id returns STATE. */
 int rafd_step_group(rafd_room **rooms, int32_t n, int64_t nsteps);
 
+/* Cross-process slabs without NCCL: a slab created with
+ * nranks > 1 and nccl_id = NULL exports a RAFD_IPC_BLOB_BYTES blob (CUDA IPC
+ * handles of its two field buffers and its two 64-bit signal words, plus its
+ * plane count and pitch); the caller exchanges blobs (e.g. torch.distributed
+ * all_gather_object) and connects each slab to its neighbours' blobs (NULL at
+ * the room's ends).  Afterwards rafd_step runs the edge-first step with the
+ * halo planes pulled by device-to-device (peer) copies, ordered by GPU-side
+ * stream waits on the neighbours' signal words -- no host round trip, no NCCL.
+ * Neighbours may be on the same GPU or on peer GPUs (NVLink).  All slabs must
+ * step the same number of times.  Errors: STATE, INVAL, CUDA. */
+#define RAFD_IPC_BLOB_BYTES 208
+int rafd_ipc_handle(rafd_room *r, uint8_t *blob);
+int rafd_ipc_connect(rafd_room *r, const uint8_t *lower, const uint8_t *upper);
+
 /* Wait for all enqueued work of the room. */
 int rafd_synchronize(rafd_room *r);
 

@@ -142,3 +142,171 @@ cudaError_t halo_exchange(Halo *h, void *buf, size_t plane_bytes, int lnz, cudaS
 }
 
 }  // namespace rafd
+
+// ================================================================ IPC transport
+#include <cudaTypedefs.h>
+
+namespace rafd {
+
+struct IpcPeer {
+    void *u[2] = {nullptr, nullptr};
+    int64_t *sig = nullptr;
+    bool open = false;
+    int lnz = 0;
+    uint32_t pitch = 0;
+};
+
+struct HaloIpc {
+    IpcPeer lo, hi;
+};
+
+static const uint32_t kMagic = 0x52414644u;  // "RAFD"
+
+struct StreamMemOps {
+    PFN_cuStreamWaitValue32_v2 wait = nullptr;
+    PFN_cuStreamWriteValue32_v2 write = nullptr;
+    bool ok = false;
+};
+
+static StreamMemOps &memops()
+{
+    static StreamMemOps m;
+    static bool tried = false;
+    if (!tried) {
+        tried = true;
+        cudaDriverEntryPointQueryResult q;
+        void *p = nullptr;
+        if (cudaGetDriverEntryPoint("cuStreamWaitValue32", &p, cudaEnableDefault, &q) == cudaSuccess &&
+            q == cudaDriverEntryPointSuccess)
+            m.wait = (PFN_cuStreamWaitValue32_v2)p;
+        p = nullptr;
+        if (cudaGetDriverEntryPoint("cuStreamWriteValue32", &p, cudaEnableDefault, &q) == cudaSuccess &&
+            q == cudaDriverEntryPointSuccess)
+            m.write = (PFN_cuStreamWriteValue32_v2)p;
+        m.ok = m.wait && m.write;
+        if (!m.ok) h_err = "cuStreamWaitValue32/cuStreamWriteValue32 unavailable";
+    }
+    return m;
+}
+
+int ipc_make_blob(void *u0, void *u1, int64_t *sig, int device, int lnz, uint32_t pitch, uint8_t *blob)
+{
+    cudaIpcMemHandle_t h[3];
+    void *p[3] = {u0, u1, sig};
+    for (int k = 0; k < 3; k++) {
+        cudaError_t e = cudaIpcGetMemHandle(&h[k], p[k]);
+        if (e != cudaSuccess) {
+            h_err = std::string("cudaIpcGetMemHandle: ") + cudaGetErrorString(e);
+            return RAFD_E_CUDA;
+        }
+        memcpy(blob + 64 * k, &h[k], 64);
+    }
+    uint32_t tail[4] = {kMagic, (uint32_t)device, (uint32_t)lnz, pitch};
+    memcpy(blob + 192, tail, 16);
+    return RAFD_OK;
+}
+
+static int open_peer(IpcPeer &pe, const uint8_t *blob)
+{
+    uint32_t tail[4];
+    memcpy(tail, blob + 192, 16);
+    if (tail[0] != kMagic) {
+        h_err = "not a rafd IPC blob";
+        return RAFD_E_INVAL;
+    }
+    pe.lnz = (int)tail[2];
+    pe.pitch = tail[3];
+    void **dst[3] = {&pe.u[0], &pe.u[1], (void **)&pe.sig};
+    for (int k = 0; k < 3; k++) {
+        cudaIpcMemHandle_t h;
+        memcpy(&h, blob + 64 * k, 64);
+        cudaError_t e = cudaIpcOpenMemHandle(dst[k], h, cudaIpcMemLazyEnablePeerAccess);
+        if (e != cudaSuccess) {
+            h_err = std::string("cudaIpcOpenMemHandle: ") + cudaGetErrorString(e);
+            return RAFD_E_CUDA;
+        }
+    }
+    pe.open = true;
+    return RAFD_OK;
+}
+
+int ipc_open(HaloIpc **out, const uint8_t *lower, const uint8_t *upper, uint32_t pitch)
+{
+    *out = nullptr;
+    for (const uint8_t *b : {lower, upper}) {
+        if (!b) continue;
+        uint32_t tail[4];
+        memcpy(tail, b + 192, 16);
+        if (tail[0] != kMagic || tail[3] != pitch) {
+            h_err = "IPC blob is not a slab of the same room (magic / pitch mismatch)";
+            return RAFD_E_INVAL;
+        }
+    }
+    if (!memops().ok) return RAFD_E_CUDA;
+    HaloIpc *h = new HaloIpc();
+    int rc = RAFD_OK;
+    if (lower) rc = open_peer(h->lo, lower);
+    if (!rc && upper) rc = open_peer(h->hi, upper);
+    if (rc) {
+        ipc_close(h);
+        return rc;
+    }
+    *out = h;
+    return RAFD_OK;
+}
+
+void ipc_close(HaloIpc *h)
+{
+    if (!h) return;
+    for (IpcPeer *pe : {&h->lo, &h->hi}) {
+        if (!pe->open) continue;
+        for (int k = 0; k < 2; k++)
+            if (pe->u[k]) cudaIpcCloseMemHandle(pe->u[k]);
+        if (pe->sig) cudaIpcCloseMemHandle(pe->sig);
+    }
+    delete h;
+}
+
+// 32-bit stream memory operations (64-bit ones need an optional device
+// capability); step counters stay far below 2^31.
+cudaError_t ipc_signal(int64_t *addr, int64_t value, cudaStream_t s)
+{
+    // default flags: ordered after prior work in the stream, with a memory barrier
+    CUresult r = memops().write((CUstream)s, (CUdeviceptr)addr, (cuuint32_t)value, CU_STREAM_WRITE_VALUE_DEFAULT);
+    if (r != CUDA_SUCCESS) {
+        h_err = "cuStreamWriteValue32 failed (CUresult " + std::to_string((int)r) + ")";
+        return cudaErrorUnknown;
+    }
+    return cudaSuccess;
+}
+
+cudaError_t ipc_wait_peers(HaloIpc *h, int word, int64_t value, cudaStream_t s)
+{
+    for (IpcPeer *pe : {&h->lo, &h->hi}) {
+        if (!pe->open) continue;
+        CUresult r = memops().wait((CUstream)s, (CUdeviceptr)(pe->sig + word), (cuuint32_t)value,
+                                   CU_STREAM_WAIT_VALUE_GEQ);
+        if (r != CUDA_SUCCESS) {
+            h_err = "cuStreamWaitValue32 failed (CUresult " + std::to_string((int)r) + ")";
+            return cudaErrorUnknown;
+        }
+    }
+    return cudaSuccess;
+}
+
+// ghost planes of my buffer `buf` <- the neighbours' edge planes of their buffer `buf`
+// (all slabs step in lock-step, so they use the same buffer parity)
+cudaError_t ipc_pull(HaloIpc *h, int buf, void *mine, size_t plane_bytes, int lnz, cudaStream_t s)
+{
+    char *m = (char *)mine;
+    cudaError_t e = cudaSuccess;
+    if (h->lo.open)
+        e = cudaMemcpyAsync(m, (const char *)h->lo.u[buf] + (size_t)h->lo.lnz * plane_bytes, plane_bytes,
+                            cudaMemcpyDeviceToDevice, s);
+    if (e == cudaSuccess && h->hi.open)
+        e = cudaMemcpyAsync(m + (size_t)(lnz + 1) * plane_bytes, (const char *)h->hi.u[buf] + plane_bytes,
+                            plane_bytes, cudaMemcpyDeviceToDevice, s);
+    return e;
+}
+
+}  // namespace rafd

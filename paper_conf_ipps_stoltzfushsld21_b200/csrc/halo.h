@@ -17,3 +17,24 @@ cudaError_t halo_exchange(Halo *h, void *buf, size_t plane_bytes, int lnz, cudaS
 int halo_unique_id(uint8_t *id128);
 const char *halo_last_error();
 }  // namespace rafd
+
+// ---------------------------------------------------------------- IPC transport
+// Slabs in different processes (same or peer GPUs): each rank maps its
+// neighbours' two field buffers and 16-byte signal words via CUDA IPC, copies
+// the neighbours' edge planes into its ghost planes with device-to-device
+// copies, and orders everything with GPU-side stream memory operations
+// (cuStreamWriteValue64 / cuStreamWaitValue64 on the signal words): no host
+// round trip, no NCCL.  Signal word 0 = "edge planes of step n done" (n+1),
+// word 1 = "my copies out of my neighbours' buffers for step n done" (n+1).
+namespace rafd {
+struct HaloIpc;
+constexpr int kIpcBlobBytes = 3 * 64 + 16;
+// blob of this rank: IPC handles of u0, u1, sig + (magic, device, lnz, pitch)
+int ipc_make_blob(void *u0, void *u1, int64_t *sig, int device, int lnz, uint32_t pitch, uint8_t *blob);
+int ipc_open(HaloIpc **out, const uint8_t *lower, const uint8_t *upper, uint32_t pitch);
+void ipc_close(HaloIpc *h);
+// per-step pieces (stream-ordered)
+cudaError_t ipc_signal(int64_t *addr, int64_t value, cudaStream_t s);
+cudaError_t ipc_wait_peers(HaloIpc *h, int word, int64_t value, cudaStream_t s);
+cudaError_t ipc_pull(HaloIpc *h, int buf, void *mine, size_t plane_bytes, int lnz, cudaStream_t s);
+}  // namespace rafd

@@ -112,6 +112,8 @@ struct rafd_room {
     // process (rafd_step_group), device-to-device / peer copies
     Halo *halo = nullptr;
     bool local_slab = false;
+    HaloIpc *ipc = nullptr;   // cross-process slabs (rafd_ipc_connect)
+    int64_t *ipc_sig = nullptr;  // [2] IPC signal words (edge done, pulls done)
     // edge-first step of a slab: edge planes, then the halo exchange on
     // comm_stream overlapped with the interior planes
     cudaStream_t comm_stream = nullptr;
@@ -407,6 +409,8 @@ extern "C" int rafd_create(const rafd_room_desc *d, rafd_room **out)
     }
     if (d->device < 0 || d->device >= ndev) return set_err(RAFD_E_INVAL, "device %d out of range", d->device);
     CK(cudaSetDevice(d->device));
+    // L2 fetch granularity (experiment knob; device-wide, so opt-in only)
+    if (const char *lf = getenv("RAFD_L2_FETCH")) cudaDeviceSetLimit(cudaLimitMaxL2FetchGranularity, (size_t)atoi(lf));
     rafd_room *r = new rafd_room();
     r->device = d->device;
     r->prec = d->precision;
@@ -446,6 +450,7 @@ extern "C" int rafd_create(const rafd_room_desc *d, rafd_room **out)
             r->local_slab = true;  // stepped by rafd_step_group in this process
         }
         cudaStreamCreateWithFlags(&r->comm_stream, cudaStreamNonBlocking);
+        if (!rc && cudaMalloc((void **)&r->ipc_sig, 64) == cudaSuccess) cudaMemset(r->ipc_sig, 0, 64);
         cudaEventCreateWithFlags(&r->ev_edge, cudaEventDisableTiming);
         cudaEventCreateWithFlags(&r->ev_halo, cudaEventDisableTiming);
     }
@@ -475,6 +480,8 @@ extern "C" void rafd_destroy(rafd_room *r)
     if (r->stream) cudaStreamSynchronize(r->stream);
     free_graphs(r);
     if (r->halo) halo_destroy(r->halo);
+    if (r->ipc) ipc_close(r->ipc);
+    if (r->ipc_sig) cudaFree(r->ipc_sig);
     if (r->ev_edge) cudaEventDestroy(r->ev_edge);
     if (r->ev_halo) cudaEventDestroy(r->ev_halo);
     if (r->comm_stream) cudaStreamDestroy(r->comm_stream);
@@ -739,6 +746,25 @@ static int kernels_per_phase(const rafd_room *r, int phase)
     return (lnz > 2 ? 1 : 0) + nbk * (lnz > 2 && r->n_last_start > r->n_first_plane ? 1 : 0) + 1;
 }
 
+// one IPC-halo step of this rank (step index n since creation)
+template <typename T> static cudaError_t enqueue_step_ipc(rafd_room *r, bool prof, int64_t n)
+{
+    cudaError_t e = cudaSuccess;
+    if (n > 0 && (e = ipc_wait_peers(r->ipc, 1, n, r->stream)) != cudaSuccess) return e;  // WAR on my edge planes
+    if ((e = enqueue_phase<T>(r, 0, r->stream, prof)) != cudaSuccess) return e;
+    if ((e = ipc_signal(r->ipc_sig + 0, n + 1, r->stream)) != cudaSuccess) return e;
+    if ((e = cudaEventRecord(r->ev_edge, r->stream)) != cudaSuccess) return e;
+    if ((e = cudaStreamWaitEvent(r->comm_stream, r->ev_edge, 0)) != cudaSuccess) return e;
+    if ((e = ipc_wait_peers(r->ipc, 0, n + 1, r->comm_stream)) != cudaSuccess) return e;
+    if ((e = ipc_pull(r->ipc, r->cur ^ 1, r->u[r->cur ^ 1], (size_t)r->g.plane * sizeof(T), r->g.lnz, r->comm_stream)) !=
+        cudaSuccess)
+        return e;
+    if ((e = ipc_signal(r->ipc_sig + 1, n + 1, r->comm_stream)) != cudaSuccess) return e;
+    if ((e = cudaEventRecord(r->ev_halo, r->comm_stream)) != cudaSuccess) return e;
+    if ((e = enqueue_phase<T>(r, 1, r->stream, prof)) != cudaSuccess) return e;
+    return cudaStreamWaitEvent(r->stream, r->ev_halo, 0);
+}
+
 // one NCCL-halo step of this rank
 template <typename T> static cudaError_t enqueue_step_nccl(rafd_room *r, bool prof)
 {
@@ -777,7 +803,7 @@ template <typename T> static int step_t(rafd_room *r, int64_t nsteps)
     if (rc) return rc;
     const int kps = kernels_per_step(r);
     int64_t done = 0;
-    const bool use_graph = !r->profiling && !r->halo && nsteps >= rafd_room::G;
+    const bool use_graph = !r->profiling && !r->halo && !r->ipc && nsteps >= rafd_room::G;
     while (use_graph && nsteps - done >= rafd_room::G) {
         if (!r->graph[r->cur] && (rc = build_graph<T>(r, r->cur))) return rc;
         CK(cudaGraphLaunch(r->graph[r->cur], r->stream));
@@ -789,6 +815,10 @@ template <typename T> static int step_t(rafd_room *r, int64_t nsteps)
         if (r->halo) {
             e = enqueue_step_nccl<T>(r, r->profiling);
             if (e == cudaErrorUnknown) return set_err(RAFD_E_NCCL, "%s", halo_last_error());
+            r->launches += kernels_per_phase(r, 0) + kernels_per_phase(r, 1);
+        } else if (r->ipc) {
+            e = enqueue_step_ipc<T>(r, r->profiling, r->steps + done);
+            if (e == cudaErrorUnknown) return set_err(RAFD_E_CUDA, "%s", halo_last_error());
             r->launches += kernels_per_phase(r, 0) + kernels_per_phase(r, 1);
         } else {
             e = enqueue_step<T>(r, r->cur, r->stream, r->profiling);
@@ -805,7 +835,8 @@ template <typename T> static int step_t(rafd_room *r, int64_t nsteps)
 extern "C" int rafd_step(rafd_room *r, int64_t nsteps)
 {
     if (!r || nsteps < 0) return set_err(RAFD_E_INVAL, "bad step arguments");
-    if (r->local_slab) return set_err(RAFD_E_STATE, "a slab created without nccl_id is stepped with rafd_step_group");
+    if (r->local_slab && !r->ipc)
+        return set_err(RAFD_E_STATE, "a slab created without nccl_id is stepped with rafd_step_group or after rafd_ipc_connect");
     if (nsteps == 0) return RAFD_OK;
     CK(cudaSetDevice(r->device));
     return r->prec == 32 ? step_t<float>(r, nsteps) : step_t<double>(r, nsteps);
@@ -908,6 +939,30 @@ extern "C" int rafd_step_group(rafd_room **rooms, int32_t n, int64_t nsteps)
         }
     }
     return rooms[0]->prec == 32 ? step_group_t<float>(rooms, n, nsteps) : step_group_t<double>(rooms, n, nsteps);
+}
+
+extern "C" int rafd_ipc_handle(rafd_room *r, uint8_t *blob)
+{
+    if (!r || !blob) return set_err(RAFD_E_INVAL, "bad arguments");
+    if (!r->local_slab || !r->ipc_sig) return set_err(RAFD_E_STATE, "IPC handles exist for slabs created without nccl_id");
+    CK(cudaSetDevice(r->device));
+    int rc = ipc_make_blob(r->u[0], r->u[1], r->ipc_sig, r->device, r->g.lnz, (uint32_t)r->g.pitch, blob);
+    if (rc) return set_err(rc, "%s", halo_last_error());
+    return RAFD_OK;
+}
+
+extern "C" int rafd_ipc_connect(rafd_room *r, const uint8_t *lower, const uint8_t *upper)
+{
+    if (!r) return set_err(RAFD_E_INVAL, "null room");
+    if (!r->local_slab || r->ipc) return set_err(RAFD_E_STATE, "rafd_ipc_connect: not an unconnected slab");
+    if ((r->rank > 0) != (lower != nullptr) || (r->rank < r->nranks - 1) != (upper != nullptr))
+        return set_err(RAFD_E_INVAL, "rank %d of %d needs %s lower and %s upper neighbour", r->rank, r->nranks,
+                       r->rank > 0 ? "a" : "no", r->rank < r->nranks - 1 ? "an" : "no");
+    CK(cudaSetDevice(r->device));
+    CK(cudaStreamSynchronize(r->stream));
+    int rc = ipc_open(&r->ipc, lower, upper, (uint32_t)r->g.pitch);
+    if (rc) return set_err(rc, "%s", halo_last_error());
+    return RAFD_OK;
 }
 
 extern "C" int rafd_synchronize(rafd_room *r)

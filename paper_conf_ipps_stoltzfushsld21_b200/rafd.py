@@ -37,7 +37,9 @@ ABI_SYMBOLS = [
     "rafd_read_branch_state", "rafd_get_classification", "rafd_get_info", "rafd_energy",
     "rafd_set_profiling", "rafd_get_kernel_times", "rafd_launch_count", "rafd_slab_plan",
     "rafd_nccl_unique_id", "rafd_last_error", "rafd_strerror", "rafd_version",
+    "rafd_ipc_handle", "rafd_ipc_connect",
 ]
+RAFD_IPC_BLOB_BYTES = 208
 
 
 class rafd_materials(C.Structure):
@@ -107,6 +109,8 @@ def lib():
     L.rafd_launch_count.restype = I64
     L.rafd_slab_plan.argtypes = [I32, I32, I32, P, I32, I32, I32, P, P]
     L.rafd_nccl_unique_id.argtypes = [P]
+    L.rafd_ipc_handle.argtypes = [P, P]
+    L.rafd_ipc_connect.argtypes = [P, P, P]
     L.rafd_last_error.restype = C.c_char_p
     L.rafd_strerror.restype = C.c_char_p
     L.rafd_strerror.argtypes = [C.c_int]
@@ -286,6 +290,18 @@ class Room:
         t = rafd_kernel_times()
         _check(lib().rafd_get_kernel_times(self.h, C.byref(t)))
         return {k: getattr(t, k) for k, _ in rafd_kernel_times._fields_}
+
+    def ipc_handle(self):
+        """This slab's IPC blob (bytes) for rafd_ipc_connect of its neighbours."""
+        buf = (C.c_uint8 * RAFD_IPC_BLOB_BYTES)()
+        _check(lib().rafd_ipc_handle(self.h, buf))
+        return bytes(buf)
+
+    def ipc_connect(self, lower, upper):
+        lo = None if lower is None else (C.c_uint8 * RAFD_IPC_BLOB_BYTES).from_buffer_copy(lower)
+        hi = None if upper is None else (C.c_uint8 * RAFD_IPC_BLOB_BYTES).from_buffer_copy(upper)
+        _check(lib().rafd_ipc_connect(self.h, None if lo is None else C.addressof(lo),
+                                      None if hi is None else C.addressof(hi)))
 
     def launch_count(self):
         return int(lib().rafd_launch_count(self.h))
