@@ -103,7 +103,7 @@ class ClockSampler:
 def workload(cfg_name, nranks):
     cfg = dict(I.CONFIGS[cfg_name])
     nx, ny, nz = cfg["dims"]
-    if nranks > 1 and cfg_name != "C5":
+    if nranks > 1 and cfg_name != "C5" and cfg["shape"] == "box":
         nz = nz * nranks          # weak scaling: one C4-sized slab per GPU
     cfg["room"] = (nx, ny, nz)
     return cfg
@@ -114,7 +114,10 @@ def slab_inputs(cfg, z0, z1, device):
     on `device`; returns (mask, matmap, mask_z0)."""
     nx, ny, nz = cfg["room"]
     lo, hi = max(0, z0 - 1), min(nz, z1 + 1)
-    assert cfg["shape"] == "box", "bench.py generates box halls slab by slab"
+    if cfg["shape"] != "box":   # non-cuboid configs (C2): whole room, then the slab's planes
+        full = I.make_mask(cfg["shape"], nx, ny, nz, device=device)
+        mm = I.material_map(full, cfg["rule"], cfg["M"])
+        return full[lo:hi].contiguous(), mm[lo:hi].contiguous(), lo
     mask = torch.ones((hi - lo, ny, nx), dtype=torch.uint8, device=device)
     if cfg["rule"] == "region":
         mm = I.region_map_box(nx, ny, nz, lo, hi, M=cfg["M"], device=device)
@@ -206,8 +209,9 @@ def run_rafd(args, rank, world, local_rank):
     t_create = time.perf_counter() - t_c
     del mask, mm
     torch.cuda.empty_cache()
-    room.set_source(I.source_position((nx, ny, nz)), I.impulse())
-    room.set_receivers(I.receiver_positions((nx, ny, nz)))
+    mask_np = None if cfg["shape"] == "box" else I.make_mask(cfg["shape"], nx, ny, nz).numpy()
+    room.set_source(I.source_position((nx, ny, nz), mask_np), I.impulse())
+    room.set_receivers(I.receiver_positions((nx, ny, nz), mask_np))
     info = room.get_info()
 
     # warm-up (also builds the CUDA graphs)
@@ -343,7 +347,8 @@ def run_e2e(args, cfg, prec, beta0, D, E, F, rank, world, local_rank, plan, mult
         nccl_id = obj[0]
     ipc = world > 1 and args.transport == "ipc"
     sig = I.impulse()
-    rcv = I.receiver_positions((nx, ny, nz))
+    mask_np = None if cfg["shape"] == "box" else I.make_mask(cfg["shape"], nx, ny, nz).numpy()
+    rcv = I.receiver_positions((nx, ny, nz), mask_np)
     steps = args.steps
     if world > 1:
         torch.distributed.barrier()
@@ -354,7 +359,7 @@ def run_e2e(args, cfg, prec, beta0, D, E, F, rank, world, local_rank, plan, mult
                      dims=(nx, ny, nz))
     if ipc:
         connect_ipc(room, rank, world)
-    room.set_source(I.source_position((nx, ny, nz)), sig)
+    room.set_source(I.source_position((nx, ny, nz), mask_np), sig)
     room.set_receivers(rcv)
     d2h = 0
     for _ in range(steps):
@@ -385,13 +390,18 @@ def oracle_sample(cfg, nplanes):
     `nplanes` planes (a box of nx x ny x nplanes), same materials."""
     from oracle import orc
     nx, ny, nz = cfg["room"]
-    mask = I.box_mask(nx, ny, nplanes)
+    if cfg["shape"] == "box":
+        mask = I.box_mask(nx, ny, nplanes)
+    else:  # a slice of planes from the middle of the non-cuboid room
+        z0 = max(0, nz // 2 - nplanes // 2)
+        mask = I.make_mask(cfg["shape"], nx, ny, nz)[z0:z0 + nplanes].contiguous()
     mm = I.material_map(mask, cfg["rule"], cfg["M"]).numpy()
     beta0, D, E, F = I.config_materials(cfg)
     prec = cfg["precision"]
     r = orc.OracleRoom(mask.numpy(), LAM, prec, beta0, D, E, F, matmap=mm)
-    r.set_source(I.source_position((nx, ny, nplanes)), I.impulse())
-    r.set_receivers(I.receiver_positions((nx, ny, nplanes)))
+    m = mask.numpy()
+    r.set_source(I.source_position((nx, ny, nplanes), m), I.impulse())
+    r.set_receivers(I.receiver_positions((nx, ny, nplanes), m))
     return r, (nx, ny, nplanes)
 
 

@@ -75,6 +75,7 @@ template <typename T> struct FusedArgs {
     int scheme;      // 0: Listing 2 volume; 1: Listing 1 single kernel; 2: Listing 6 naive FI
     T beta1;         // Listing 1 admittance
     T loss1, loss2;  // Listing 6 constants
+    const uint8_t *occ;  // [lnz+2][tiles] tile-plane occupancy (set by the plan), or nullptr
 };
 
 // plan == nullptr selects the one-thread-per-voxel v0 kernel (A/B reference);
@@ -87,6 +88,7 @@ cudaError_t launch_volume(const Grid &g, const T *cur, T *nxt, const uint8_t *K,
                           const FusedArgs<T> *fa = nullptr);
 cudaError_t volume_plan_fuse(void *plan, const Grid &g, const uint8_t *K, int64_t Nb, cudaStream_t s);
 bool volume_plan_fused(const void *plan);
+cudaError_t volume_plan_occupancy(void *plan, const Grid &g, const uint8_t *K, cudaStream_t s);
 template <typename T>
 cudaError_t volume_plan_create(const Grid &g, void *u0, void *u1, uint8_t *K, int nsm, void **plan);
 void volume_plan_destroy(void *plan);

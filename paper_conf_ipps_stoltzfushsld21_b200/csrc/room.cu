@@ -382,7 +382,11 @@ template <typename T> static int create_t(rafd_room *r, const rafd_room_desc *d)
     c.src_pos = -1;
     CK(cudaMemcpy(r->ctl, &c, sizeof c, cudaMemcpyHostToDevice));
     const char *env = getenv("RAFD_VOLUME_KERNEL");
-    if (!(env && strcmp(env, "v0") == 0)) CK(volume_plan_create<T>(g, r->u[0], r->u[1], r->K_alloc, r->nsm, &r->vplan));
+    if (!(env && strcmp(env, "v0") == 0)) {
+        CK(volume_plan_create<T>(g, r->u[0], r->u[1], r->K_alloc, r->nsm, &r->vplan));
+        const char *sk = getenv("RAFD_SKIP_EMPTY");  // skipping of all-outside tile-planes (default on)
+        if (!(sk && strcmp(sk, "0") == 0)) CK(volume_plan_occupancy(r->vplan, g, r->K, r->stream));
+    }
     // boundary update fused into the volume kernel with RAFD_FUSED=1 (DESIGN.md
     // §6; needs the default tiling, MB <= 4, Nb < 2^31).  Off by default: the
     // first fused form is latency-bound at x-wall rows (5.6 ms vs 2.55 ms).

@@ -290,3 +290,26 @@ def test_scheme_validation():
     with pytest.raises(rafd.RafdError) as e:
         rafd.Room(mask, LAM, 32, [0.0], D=[[1.0]], E=[[1.0]], F=[[1.0]], scheme=2)
     assert e.value.code == rafd.RAFD_E_INVAL
+
+
+@pytest.mark.parametrize("shape", ["lshape", "dome"])
+def test_empty_tile_skipping_bitwise(orc, shape, monkeypatch):
+    """Tile-planes without inside voxels are skipped by the volume kernel
+    (loads, compute, store); results equal the unskipped kernel and the oracle."""
+    mask_t = I.make_mask(shape, 300, 260, 48)
+    mm = I.material_map(mask_t, "region", 8).numpy()
+    mask = mask_t.numpy()
+    beta0, D, E, F = I.fd_tables(8, 3)
+    src = I.source_position((300, 260, 48), mask)
+    out = []
+    for skip in ("1", "0"):
+        monkeypatch.setenv("RAFD_SKIP_EMPTY", skip)
+        g = rafd.Room(mask, LAM, 32, beta0, D, E, F, matmap=mm)
+        g.set_source(src, I.gaussian_pulse(40, 4.0))
+        g.step(90)
+        out.append(g.read_field()[0])
+    o = orc.OracleRoom(mask, LAM, 32, beta0, D, E, F, matmap=mm)
+    o.set_source(src, I.gaussian_pulse(40, 4.0))
+    o.step(90)
+    assert_close(o.read_field()[0], out[0], 32, "skip")
+    assert np.array_equal(out[0], out[1])
