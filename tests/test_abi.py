@@ -127,4 +127,3 @@ def test_slab_and_ipc_entry_points_reject_misuse(L):
     assert rafd.lib().rafd_ipc_connect(None, None, None) == rafd.RAFD_E_INVAL
     assert rafd.lib().rafd_step_group(None, 0, 1) == rafd.RAFD_E_INVAL
     assert rafd.lib().rafd_step(None, 1) == rafd.RAFD_E_INVAL
-    assert "rafd_step_group" in rafd.lib().rafd_last_error().decode() or True
