@@ -158,6 +158,14 @@ int rafd_set_receivers(rafd_room *r, int32_t n, const int32_t *xyz);
  * [MB][Nb] branch state (ci = b*Nb + i).  NULL => unchanged. */
 int rafd_set_state(rafd_room *r, const void *u_prev, const void *u_curr, const void *v, const void *g);
 
+/* Checkpoint / resume: the state of a room is (u^n, u^{n-1}, v, g, step
+ * counter n): read it with rafd_read_field / rafd_read_branch_state /
+ * rafd_get_info().steps, restore it into a room created from the same inputs
+ * with rafd_set_state and rafd_set_step (n indexes the source signal; the
+ * boundary copy of u^{n-1} is rebuilt by rafd_set_state).  The continued run
+ * is bitwise identical to the uninterrupted one.  STATE on a connected IPC slab. */
+int rafd_set_step(rafd_room *r, int64_t n);
+
 /* Enqueue nsteps time steps (volume kernel, boundary kernel, source,
  * receivers, rotation).  Asynchronous w.r.t. the host. */
 int rafd_step(rafd_room *r, int64_t nsteps);

@@ -1098,6 +1098,25 @@ template <typename T> static int field_in_t(rafd_room *r, const void *src, T *ds
     return rc;
 }
 
+template <typename T> static int set_step_t(rafd_room *r, int64_t n)
+{
+    Ctl<T> c;
+    int rc = pull_ctl<T>(r, c);
+    if (rc) return rc;
+    c.n = n;
+    rc = push_ctl<T>(r, c);
+    if (!rc) r->steps = n;
+    return rc;
+}
+
+extern "C" int rafd_set_step(rafd_room *r, int64_t n)
+{
+    if (!r || n < 0) return set_err(RAFD_E_INVAL, "bad arguments");
+    if (r->ipc) return set_err(RAFD_E_STATE, "the step counter of a connected IPC slab orders its signals");
+    CK(cudaSetDevice(r->device));
+    return r->prec == 32 ? set_step_t<float>(r, n) : set_step_t<double>(r, n);
+}
+
 extern "C" int rafd_set_state(rafd_room *r, const void *u_prev, const void *u_curr, const void *v, const void *g)
 {
     if (!r) return set_err(RAFD_E_INVAL, "null room");

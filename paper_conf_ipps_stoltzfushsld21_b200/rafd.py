@@ -37,7 +37,7 @@ ABI_SYMBOLS = [
     "rafd_read_branch_state", "rafd_get_classification", "rafd_get_info", "rafd_energy",
     "rafd_set_profiling", "rafd_get_kernel_times", "rafd_launch_count", "rafd_slab_plan",
     "rafd_nccl_unique_id", "rafd_last_error", "rafd_strerror", "rafd_version",
-    "rafd_ipc_handle", "rafd_ipc_connect",
+    "rafd_ipc_handle", "rafd_ipc_connect", "rafd_set_step",
 ]
 RAFD_IPC_BLOB_BYTES = 208
 
@@ -95,6 +95,7 @@ def lib():
     L.rafd_set_receivers.argtypes = [P, I32, P]
     L.rafd_set_state.argtypes = [P, P, P, P, P]
     L.rafd_step.argtypes = [P, I64]
+    L.rafd_set_step.argtypes = [P, I64]
     L.rafd_step_group.argtypes = [C.POINTER(P), I32, I64]
     L.rafd_synchronize.argtypes = [P]
     L.rafd_read_receivers.argtypes = [P, P, I64, C.POINTER(I64)]
@@ -226,6 +227,9 @@ class Room:
             return np.ascontiguousarray(a, dtype=self.dtype)
         arrs = [conv(a) for a in (u_prev, u_curr, v, g)]
         _check(lib().rafd_set_state(self.h, *[_addr(a) for a in arrs]))
+
+    def set_step(self, n):
+        _check(lib().rafd_set_step(self.h, int(n)))
 
     # --- run
     def step(self, n):

@@ -313,3 +313,35 @@ def test_empty_tile_skipping_bitwise(orc, shape, monkeypatch):
     o.step(90)
     assert_close(o.read_field()[0], out[0], 32, "skip")
     assert np.array_equal(out[0], out[1])
+
+
+@pytest.mark.parametrize("precision,MB", [(32, 3), (64, 0)])
+def test_checkpoint_resume_bitwise(precision, MB):
+    """Save (u^n, u^{n-1}, v, g, n) after 70 steps, restore into a fresh room,
+    continue 50 steps: bitwise equal to 120 uninterrupted steps (the source
+    signal continues at the restored step index)."""
+    mask = I.dome_mask(60, 50, 40).numpy()
+    mm = I.material_map(torch.from_numpy(mask), "region", 8).numpy()
+    if MB:
+        beta0, D, E, F = I.fd_tables(8, MB)
+    else:
+        beta0, D, E, F = I.fi_beta_from_alpha(np.linspace(0.1, 0.8, 8)), None, None, None
+    src = I.source_position((60, 50, 40), mask)
+    sig = I.gaussian_pulse(200, 8.0)
+    rcv = I.receiver_positions((60, 50, 40), mask)
+    a = rafd.Room(mask, LAM, precision, beta0, D, E, F, matmap=mm)
+    a.set_source(src, sig)
+    a.set_receivers(rcv)
+    a.step(70)
+    cur, prv = a.read_field()
+    v, g = a.read_branch_state() if MB else (None, None)
+    n = a.get_info()["steps"]
+    a.step(50)
+    b = rafd.Room(mask, LAM, precision, beta0, D, E, F, matmap=mm)
+    b.set_source(src, sig)
+    b.set_receivers(rcv)
+    b.set_state(prv, cur, v, g)
+    b.set_step(n)
+    b.step(50)
+    assert np.array_equal(a.read_field()[0], b.read_field()[0])
+    assert np.array_equal(a.read_receivers()[:, 70:], b.read_receivers())
