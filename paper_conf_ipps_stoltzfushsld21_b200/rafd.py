@@ -251,13 +251,14 @@ class Room:
 
     def read_field(self, out_curr=None, out_prev=None):
         """u^n and u^{n-1} of the owned planes (numpy by default; pass CUDA
-        tensors to receive on the device)."""
+        tensors to receive on the device; pass False to skip one)."""
         lnz = self.z_end - self.z_begin
         shp = (lnz, self.shape[1], self.shape[2])
         cur = np.zeros(shp, dtype=self.dtype) if out_curr is None else out_curr
         prv = np.zeros(shp, dtype=self.dtype) if out_prev is None else out_prev
-        _check(lib().rafd_read_field(self.h, _addr(cur), _addr(prv)))
-        return cur, prv
+        _check(lib().rafd_read_field(self.h, None if cur is False else _addr(cur),
+                                     None if prv is False else _addr(prv)))
+        return (None if cur is False else cur), (None if prv is False else prv)
 
     def read_branch_state(self):
         v = np.zeros((self.MB, self.nb), dtype=self.dtype)

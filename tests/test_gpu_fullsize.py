@@ -90,3 +90,39 @@ def test_config_full_size_bitwise(orc, name, precision, steps):
         vg, gg = g.read_branch_state()
         vo, go = o.read_branch_state()
         assert np.array_equal(vg, vo) and np.array_equal(gg, go)
+
+
+def test_c5_hall_int64_indexing_light_cone():
+    """The C5 hall (2048x1536x2560 = 8.05e9 voxels, fp32, FD-MM) on one GPU:
+    more than 2^32 grid elements, so boundary positions are int64.  A source
+    next to the corner (10,10,10): after 50 steps the disturbance lies within
+    50 voxels of it, so the C5 field must equal, bit for bit, that of a small
+    box with the same corner walls (its far walls are beyond the light cone)."""
+    cfg = bench.workload("C5", 1)
+    nx, ny, nz = cfg["room"]
+    beta0, D, E, F = I.config_materials(cfg)
+    dev = torch.device("cuda", 0)
+    mask, mm, _ = bench.slab_inputs(cfg, 0, nz, dev)
+    big = rafd.Room(mask, LAM, 32, beta0, D, E, F, matmap=mm)
+    del mask, mm
+    torch.cuda.empty_cache()
+    assert big.get_info()["n_boundary"] == 24616968
+    src, steps, n = (10, 10, 10), 50, 128
+    sig = I.gaussian_pulse(24, 3.0)
+    big.set_source(src, sig)
+    big.step(steps)
+    cur = torch.empty((nz, ny, nx), dtype=torch.float32, device=dev)
+    big.read_field(out_curr=cur, out_prev=False)
+    corner = cur[:n, :n, :n].cpu().numpy()
+    del cur, big
+    torch.cuda.empty_cache()
+    # the small box: same corner walls and, near the corner, the same region materials
+    small_mask = np.ones((n, n, n), np.uint8)
+    small_mm = I.region_map_box(nx, ny, nz, 0, n, device="cpu")[:, :n, :n].contiguous().numpy()
+    small = rafd.Room(small_mask, LAM, 32, beta0, D, E, F, matmap=small_mm)
+    small.set_source(src, sig)
+    small.step(steps)
+    ref = small.read_field()[0]
+    reach = 10 + steps + 1
+    assert np.array_equal(corner[:reach, :reach, :reach], ref[:reach, :reach, :reach])
+    assert np.abs(ref).max() > 1e-3 and not np.any(corner[reach:, :, :])
