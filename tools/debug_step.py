@@ -11,7 +11,8 @@ from paper_conf_ipps_stoltzfushsld21_b200 import inputs as I, rafd  # noqa: E402
 prec = int(sys.argv[1]) if len(sys.argv) > 1 else 32
 MB = int(sys.argv[2]) if len(sys.argv) > 2 else 0
 n = int(sys.argv[3]) if len(sys.argv) > 3 else 20
-mask = I.dome_mask(n + 7, n + 3, n).numpy()
+shape = sys.argv[4] if len(sys.argv) > 4 else "dome"
+mask = I.make_mask(shape, 3 * n + 7, 2 * n + 3, n).numpy()
 if MB:
     b0, D, E, F = I.fd_tables(2, MB)
 else:
