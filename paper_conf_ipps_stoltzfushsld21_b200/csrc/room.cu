@@ -89,6 +89,8 @@ struct rafd_room {
     int64_t *rcv_pos = nullptr;
     void *rec = nullptr;
     int64_t rec_cap = 0, rec_count = 0;
+    void *rec_host = nullptr;  // pinned staging for rafd_read_receivers
+    size_t rec_host_bytes = 0;
     int32_t nrcv = 0;
     int64_t steps = 0;
     int64_t k_hist[7] = {0};
@@ -499,6 +501,7 @@ extern "C" void rafd_destroy(rafd_room *r)
         cudaEventDestroy(e.b);
     }
     for (auto e : r->ev_pool) cudaEventDestroy(e);
+    if (r->rec_host) cudaFreeHost(r->rec_host);
     if (r->cap_stream) cudaStreamDestroy(r->cap_stream);
     if (r->own_stream && r->stream) cudaStreamDestroy(r->stream);
     cudaGetLastError();
@@ -978,24 +981,34 @@ extern "C" int rafd_synchronize(rafd_room *r)
 }
 
 // ------------------------------------------------------------------ reads
+// One stream-ordered D2H of the unread rows into a pinned staging buffer, a
+// device-side reset of the row counter, one synchronisation (the host already
+// knows how many rows the device wrote).
 template <typename T> static int read_receivers_t(rafd_room *r, double *out, int64_t cap, int64_t *nw)
 {
-    CK(cudaStreamSynchronize(r->stream));
     const int64_t n = r->rec_count;
     if (r->nrcv > 0 && (cap < n || !out)) return set_err(RAFD_E_INVAL, "cap (%lld) < unread samples (%lld)", (long long)cap, (long long)n);
+    const size_t bytes = (size_t)n * r->nrcv * sizeof(T);
     if (r->nrcv > 0 && n > 0) {
-        std::vector<T> h((size_t)n * r->nrcv);
-        CK(cudaMemcpy(h.data(), r->rec, h.size() * sizeof(T), cudaMemcpyDeviceToHost));
+        if (r->rec_host_bytes < bytes) {
+            if (r->rec_host) cudaFreeHost(r->rec_host);
+            r->rec_host = nullptr;
+            r->rec_host_bytes = 0;
+            CK(cudaMallocHost(&r->rec_host, bytes));
+            r->rec_host_bytes = bytes;
+        }
+        CK(cudaMemcpyAsync(r->rec_host, r->rec, bytes, cudaMemcpyDeviceToHost, r->stream));
+    }
+    CK(cudaMemsetAsync(&ctl_of<T>(r)->rec_count, 0, sizeof(int64_t), r->stream));
+    CK(cudaStreamSynchronize(r->stream));
+    if (r->nrcv > 0 && n > 0) {
+        const T *h = (const T *)r->rec_host;
         for (int j = 0; j < r->nrcv; j++)
             for (int64_t k = 0; k < n; k++) out[j * cap + k] = (double)h[(size_t)k * r->nrcv + j];
     }
     *nw = r->nrcv > 0 ? n : 0;
     r->rec_count = 0;
-    Ctl<T> c;
-    int rc = pull_ctl<T>(r, c);
-    if (rc) return rc;
-    c.rec_count = 0;
-    return push_ctl<T>(r, c);
+    return RAFD_OK;
 }
 
 extern "C" int rafd_read_receivers(rafd_room *r, double *out, int64_t cap, int64_t *n_written)
