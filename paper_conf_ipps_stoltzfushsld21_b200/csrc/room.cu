@@ -60,6 +60,23 @@ static bool is_device_ptr(const void *p)
     return a.type == cudaMemoryTypeDevice || a.type == cudaMemoryTypeManaged;
 }
 
+// A pointer kernels can dereference: device / managed memory as is, pinned
+// (page-locked) host memory through its mapped device address (zero-copy over
+// PCIe: a kernel then reads exactly the bytes it needs); nullptr for pageable
+// host memory (staged through a device buffer instead).
+static const void *device_view(const void *p)
+{
+    if (!p) return nullptr;
+    cudaPointerAttributes a;
+    if (cudaPointerGetAttributes(&a, p) != cudaSuccess) {
+        cudaGetLastError();
+        return nullptr;
+    }
+    if (a.type == cudaMemoryTypeDevice || a.type == cudaMemoryTypeManaged) return p;
+    if (a.type == cudaMemoryTypeHost && a.devicePointer) return a.devicePointer;
+    return nullptr;
+}
+
 // ------------------------------------------------------------------ the room
 struct rafd_room {
     int device = 0;
@@ -281,14 +298,16 @@ template <typename T> static int create_t(rafd_room *r, const rafd_room_desc *d)
     for (int k = 0; k < 2; k++) CK(cudaMemsetAsync(r->u[k], 0, (size_t)g.total * sizeof(T) + 64, r->stream));
 
     // ---- classification (row a1)
-    const bool mdev = is_device_ptr(d->mask);
+    // the mask is streamed in full (DMA staging beats zero-copy reads for it);
+    // the matmap is only sampled at boundary nodes, so pinned host memory is
+    // read in place by the gather kernel
+    const void *mask_dv = is_device_ptr(d->mask) ? d->mask : nullptr, *matmap_dv = device_view(d->matmap);
+    const bool mdev = mask_dv != nullptr;
     void *staging = nullptr;
-    if ((!mdev || (d->matmap && !is_device_ptr(d->matmap))) &&
-        (rc = dmalloc(r, &staging, kStagingBytes)))
-        return rc;
+    if ((!mdev || (d->matmap && !matmap_dv)) && (rc = dmalloc(r, &staging, kStagingBytes))) return rc;
     const int zlo = std::max(0, r->z0 - 1), zhi = std::min(r->nz, r->z1 + 1);  // incl. ghost planes
     const int mz0 = d->mask_z0;
-    rc = for_plane_chunks(r, d->mask, mz0, mdev, (size_t)nxny, zlo, zhi - zlo, staging, kStagingBytes,
+    rc = for_plane_chunks(r, mdev ? mask_dv : d->mask, mz0, mdev, (size_t)nxny, zlo, zhi - zlo, staging, kStagingBytes,
                           [&](const void *chunk, int zg, int n) -> int {
                               CK(launch_scatter_mask(g, (const uint8_t *)chunk, zg - r->z0 + 1, n, r->K, r->stream));
                               return RAFD_OK;
@@ -343,8 +362,9 @@ template <typename T> static int create_t(rafd_room *r, const rafd_room_desc *d)
     unsigned *bad = (unsigned *)(hist + 8);
     if (!d->matmap) {
         CK(cudaMemsetAsync(r->matb, 0, (size_t)nb + 1, r->stream));
-    } else if (is_device_ptr(d->matmap)) {
-        CK(launch_gather_mat(d->matmap, (int64_t)mz0 * nxny, r->bidx, 0, nb, r->matb, r->M, bad, r->stream));
+    } else if (matmap_dv) {  // device memory, or pinned host memory read in place
+        CK(launch_gather_mat((const uint8_t *)matmap_dv, (int64_t)mz0 * nxny, r->bidx, 0, nb, r->matb, r->M, bad,
+                             r->stream));
     } else {
         std::vector<int64_t> off_h((size_t)rows + 1);
         CK(cudaMemcpyAsync(off_h.data(), row_off, (size_t)(rows + 1) * 8, cudaMemcpyDeviceToHost, r->stream));
