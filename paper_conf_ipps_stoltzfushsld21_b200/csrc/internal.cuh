@@ -32,14 +32,18 @@ template <> struct rn<double> {
 // Padded grid in HBM: (lnz+2) planes x (ny+2) rows x pitch
 // elements.  Room voxel (x, y, zl) (zl slab-local, 0..lnz-1) lives at
 //   (zl+1)*plane + (y+1)*pitch + xo + x
-// with xo = 16/sizeof(T) so every interior row starts 16-byte aligned; the x
-// halo cells are xo-1 and xo+nx; pitch is a multiple of 128 bytes.  The uint8
-// K grid uses the same element indexing.
+// with xo = 128/sizeof(T) so every interior row starts on a 128-byte line
+// (a tile's u^{n-1} reads and u+ stores then cover whole sectors, never a
+// sector shared with the neighbouring tile); the x halo cells are xo-1 and
+// xo+nx; pitch is a multiple of 128 bytes.  The uint8 K grid uses the same
+// element indexing, shifted by k_shift(g) bytes from its allocation so that
+// element xo of every row is 16-byte aligned (TMA box origin).
 struct Grid {
     int32_t nx, ny, lnz;
     int32_t xo;
     int64_t pitch, plane, total;
 };
+static inline __host__ __device__ int k_shift(const Grid &g) { return (16 - g.xo % 16) % 16; }
 
 // Device control block for the per-step source / receivers (read by the
 // src/rcv kernel so that CUDA graphs never need re-capturing).

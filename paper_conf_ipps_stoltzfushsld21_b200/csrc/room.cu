@@ -279,7 +279,7 @@ template <typename T> static int create_t(rafd_room *r, const rafd_room_desc *d)
     g.nx = r->nx;
     g.ny = r->ny;
     g.lnz = r->z1 - r->z0;
-    g.xo = (int)(16 / sizeof(T));
+    g.xo = (int)(128 / sizeof(T));
     const int64_t align = 128 / (int64_t)sizeof(T);
     g.pitch = ((g.xo + r->nx + 1 + align - 1) / align) * align;
     g.plane = g.pitch * (r->ny + 2);
@@ -288,10 +288,10 @@ template <typename T> static int create_t(rafd_room *r, const rafd_room_desc *d)
 
     int rc;
     // K grid: element (row, xo + x) must sit at a 16-byte aligned byte address
-    // for the TMA boxes of the volume kernel, so the buffer starts 16 - xo bytes
-    // before the first element (r->K_alloc is what cudaMalloc returned).
+    // for the TMA boxes of the volume kernel, so the buffer starts k_shift(g)
+    // bytes before the first element (r->K_alloc is what cudaMalloc returned).
     if ((rc = dmalloc(r, (void **)&r->K_alloc, (size_t)g.total + 64))) return rc;
-    r->K = r->K_alloc + (16 - g.xo);
+    r->K = r->K_alloc + k_shift(g);
     for (int k = 0; k < 2; k++)
         if ((rc = dmalloc(r, &r->u[k], (size_t)g.total * sizeof(T) + 64))) return rc;
     CK(cudaMemsetAsync(r->K_alloc, 0, (size_t)g.total + 64, r->stream));
