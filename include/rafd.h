@@ -134,7 +134,7 @@ typedef struct rafd_kernel_times {
 /* Create a room: validates lambda / tables / dims, copies mask and matmap to
  * the device, classifies voxels on the device (K, ascending boundary list,
  * K_b, mat_b: PAPER.md:306-323, 390-393, 411-412), allocates and zeroes the
- * two field buffers, ub_prev and the branch state.  Errors: INVAL, UNSTABLE,
+ * two field buffers, the boundary-node ring u_b and the branch state.  Errors: INVAL, UNSTABLE,
  * NONPASSIVE, MATERIAL, NOMEM, CUDA, NCCL.  *out is NULL on error. */
 int rafd_create(const rafd_room_desc *d, rafd_room **out);
 

@@ -55,6 +55,7 @@ template <typename T> struct Ctl {
     const T *sig;       // [sig_len]
     int64_t sig_len;
     int64_t src_pos;    // padded index or -1
+    int64_t src_node;   // boundary-node index of the source voxel or -1 (its u_b slot is updated too)
     int32_t nrcv;
     int32_t pad_;
     const int64_t *rcv_pos;  // [nrcv] padded indices
@@ -99,10 +100,11 @@ void volume_plan_destroy(void *plan);
 template <typename T>
 cudaError_t launch_boundary(int MB, bool idx64, const void *bpos, const uint8_t *Kb,
                             const uint8_t *matb, int64_t i_lo, int64_t i_hi, int64_t Nb, T *unext,
-                            const T *ucur, T *ub_prev, T *g, T *v, const T *tab, int M,
-                            double lambda, cudaStream_t s);
+                            T *ub, T *g, T *v, const T *tab, int M, double lambda, cudaStream_t s);
 template <typename T>
-cudaError_t launch_src_rcv(T *unext, Ctl<T> *ctl, cudaStream_t s, int mode = 3);
+cudaError_t launch_src_rcv(T *unext, T *ub, Ctl<T> *ctl, cudaStream_t s, int mode = 3);
+cudaError_t launch_find_node(const void *bpos, bool idx64, int64_t Nb, int64_t pos, int64_t *out,
+                             cudaStream_t s);
 
 // classification: flags -> K (in place, bit 7 trick), counts, compaction
 cudaError_t launch_scatter_mask(const Grid &g, const uint8_t *mask_chunk, int zp0, int nzc,

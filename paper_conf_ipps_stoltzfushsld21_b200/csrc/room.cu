@@ -147,6 +147,12 @@ struct rafd_room {
 };
 
 template <typename T> static Ctl<T> *ctl_of(rafd_room *r) { return (Ctl<T> *)r->ctl; }
+// the u_b slot of a step whose u^n is u[cur] (null when the boundary update is
+// fused into the volume kernel or a single-kernel scheme runs: no ring then)
+template <typename T> static T *ub_slot(rafd_room *r, int cur)
+{
+    return (r->fused || r->scheme || r->nb == 0) ? nullptr : (T *)r->ub + (int64_t)cur * r->nb;
+}
 
 template <typename T> static FusedArgs<T> fused_args(const rafd_room *r)
 {
@@ -350,10 +356,10 @@ template <typename T> static int create_t(rafd_room *r, const rafd_room_desc *d)
     if ((rc = dmalloc(r, (void **)&r->bidx, (size_t)nb * 8))) return rc;
     if ((rc = dmalloc(r, (void **)&r->Kb, (size_t)nb))) return rc;
     if ((rc = dmalloc(r, (void **)&r->matb, (size_t)nb))) return rc;
-    if ((rc = dmalloc(r, &r->ub, (size_t)nb * sizeof(T)))) return rc;
+    if ((rc = dmalloc(r, &r->ub, (size_t)2 * nb * sizeof(T)))) return rc;  // [2][Nb] ring, slot = cur
     if ((rc = dmalloc(r, &r->gst, (size_t)nb * r->MB * sizeof(T)))) return rc;
     if ((rc = dmalloc(r, &r->vst, (size_t)nb * r->MB * sizeof(T)))) return rc;
-    CK(cudaMemsetAsync(r->ub, 0, (size_t)nb * sizeof(T) + 16, r->stream));
+    CK(cudaMemsetAsync(r->ub, 0, (size_t)2 * nb * sizeof(T) + 16, r->stream));
     CK(cudaMemsetAsync(r->gst, 0, (size_t)nb * r->MB * sizeof(T) + 16, r->stream));
     CK(cudaMemsetAsync(r->vst, 0, (size_t)nb * r->MB * sizeof(T) + 16, r->stream));
     CK(launch_compact(g, r->K, row_off, r->z0, r->ny, r->nx, r->idx64, r->bpos, r->bidx, r->Kb, r->stream));
@@ -402,6 +408,7 @@ template <typename T> static int create_t(rafd_room *r, const rafd_room_desc *d)
     if ((rc = dmalloc(r, &r->ctl, sizeof(Ctl<T>)))) return rc;
     Ctl<T> c{};
     c.src_pos = -1;
+    c.src_node = -1;
     CK(cudaMemcpy(r->ctl, &c, sizeof c, cudaMemcpyHostToDevice));
     const char *env = getenv("RAFD_VOLUME_KERNEL");
     if (!(env && strcmp(env, "v0") == 0)) {
@@ -570,6 +577,7 @@ static int set_source_t(rafd_room *r, int32_t x, int32_t y, int32_t z, const dou
     c.sig = nullptr;
     c.sig_len = 0;
     c.src_pos = -1;
+    c.src_node = -1;
     r->src_z = -1;
     if (len > 0 && owns_plane(r, z)) {
         const int64_t p = pad_pos(r, x, y, z);
@@ -583,6 +591,15 @@ static int set_source_t(rafd_room *r, int32_t x, int32_t y, int32_t z, const dou
         c.sig = (const T *)r->sig;
         c.sig_len = len;
         c.src_pos = p;
+        if (k < 6 && r->nb > 0) {  // a boundary node: its u_b slot follows the source too
+            int64_t *dn = nullptr;
+            CK(cudaMalloc(&dn, 8));
+            cudaError_t e = launch_find_node(r->bpos, r->idx64, r->nb, p, dn, r->stream);
+            if (e == cudaSuccess) e = cudaMemcpyAsync(&c.src_node, dn, 8, cudaMemcpyDeviceToHost, r->stream);
+            if (e == cudaSuccess) e = cudaStreamSynchronize(r->stream);
+            cudaFree(dn);
+            CK(e);
+        }
         r->src_z = z;
     }
     return push_ctl<T>(r, c);
@@ -696,13 +713,13 @@ template <typename T> static cudaError_t enqueue_step(rafd_room *r, int cur, cud
     if (e != cudaSuccess) return e;
     if (r->nb > 0 && !r->fused && !r->scheme) {
         e = timed(1, [&] {
-            return launch_boundary<T>(r->MB, r->idx64, r->bpos, r->Kb, r->matb, 0, r->nb, r->nb, un, uc,
-                                      (T *)r->ub, (T *)r->gst, (T *)r->vst, (const T *)r->tab, r->M,
+            return launch_boundary<T>(r->MB, r->idx64, r->bpos, r->Kb, r->matb, 0, r->nb, r->nb, un,
+                                      ub_slot<T>(r, cur), (T *)r->gst, (T *)r->vst, (const T *)r->tab, r->M,
                                       r->lambda, s);
         });
         if (e != cudaSuccess) return e;
     }
-    e = timed(2, [&] { return launch_src_rcv<T>(un, ctl_of<T>(r), s); });
+    e = timed(2, [&] { return launch_src_rcv<T>(un, ub_slot<T>(r, cur), ctl_of<T>(r), s); });
     if (e != cudaSuccess) return e;
     return cudaSuccess;
 }
@@ -738,8 +755,8 @@ template <typename T> static cudaError_t enqueue_phase(rafd_room *r, int phase, 
     auto bnd = [&](int64_t lo, int64_t hi) -> cudaError_t {
         if (hi <= lo || r->fused || r->scheme) return cudaSuccess;
         return timed(1, [&] {
-            return launch_boundary<T>(r->MB, r->idx64, r->bpos, r->Kb, r->matb, lo, hi, r->nb, un, uc,
-                                      (T *)r->ub, (T *)r->gst, (T *)r->vst, (const T *)r->tab, r->M,
+            return launch_boundary<T>(r->MB, r->idx64, r->bpos, r->Kb, r->matb, lo, hi, r->nb, un,
+                                      ub_slot<T>(r, cur), (T *)r->gst, (T *)r->vst, (const T *)r->tab, r->M,
                                       r->lambda, s);
         });
     };
@@ -751,11 +768,11 @@ template <typename T> static cudaError_t enqueue_phase(rafd_room *r, int phase, 
         if (e == cudaSuccess && lnz > 1) e = vol(lnz - 1, lnz);
         if (e == cudaSuccess) e = bnd(0, std::min(r->n_first_plane, r->nb));
         if (e == cudaSuccess && lnz > 1) e = bnd(std::max(r->n_last_start, r->n_first_plane), r->nb);
-        if (e == cudaSuccess && src_edge) e = timed(2, [&] { return launch_src_rcv<T>(un, ctl_of<T>(r), s, 1); });
+        if (e == cudaSuccess && src_edge) e = timed(2, [&] { return launch_src_rcv<T>(un, ub_slot<T>(r, cur), ctl_of<T>(r), s, 1); });
     } else {
         if (lnz > 2) e = vol(1, lnz - 1);
         if (e == cudaSuccess && lnz > 2) e = bnd(r->n_first_plane, r->n_last_start);
-        if (e == cudaSuccess) e = timed(2, [&] { return launch_src_rcv<T>(un, ctl_of<T>(r), s, src_edge ? 2 : 3); });
+        if (e == cudaSuccess) e = timed(2, [&] { return launch_src_rcv<T>(un, ub_slot<T>(r, cur), ctl_of<T>(r), s, src_edge ? 2 : 3); });
     }
     return e;
 }
@@ -1150,6 +1167,17 @@ extern "C" int rafd_set_step(rafd_room *r, int64_t n)
     return r->prec == 32 ? set_step_t<float>(r, n) : set_step_t<double>(r, n);
 }
 
+// u_b slot `slot` <- field buffer u[buf] at the boundary nodes
+static int gather_ub_slot(rafd_room *r, int buf, int slot)
+{
+    if (r->nb == 0) return RAFD_OK;
+    if (r->prec == 32)
+        CK(launch_gather_ub<float>(r->bpos, r->idx64, r->nb, (const float *)r->u[buf], (float *)r->ub + (int64_t)slot * r->nb, r->stream));
+    else
+        CK(launch_gather_ub<double>(r->bpos, r->idx64, r->nb, (const double *)r->u[buf], (double *)r->ub + (int64_t)slot * r->nb, r->stream));
+    return RAFD_OK;
+}
+
 extern "C" int rafd_set_state(rafd_room *r, const void *u_prev, const void *u_curr, const void *v, const void *g)
 {
     if (!r) return set_err(RAFD_E_INVAL, "null room");
@@ -1160,13 +1188,15 @@ extern "C" int rafd_set_state(rafd_room *r, const void *u_prev, const void *u_cu
         rc = r->prec == 32 ? field_in_t<float>(r, u_prev, (float *)r->u[r->cur ^ 1])
                            : field_in_t<double>(r, u_prev, (double *)r->u[r->cur ^ 1]);
         if (rc) return rc;
-        // ub_prev = u^{n-1} at the boundary nodes (reading R8)
-        if (r->prec == 32) CK(launch_gather_ub<float>(r->bpos, r->idx64, r->nb, (const float *)r->u[r->cur ^ 1], (float *)r->ub, r->stream));
-        else CK(launch_gather_ub<double>(r->bpos, r->idx64, r->nb, (const double *)r->u[r->cur ^ 1], (double *)r->ub, r->stream));
+        // u_b slot cur = u^{n-1} at the boundary nodes (reading R8)
+        rc = gather_ub_slot(r, r->cur ^ 1, r->cur);
+        if (rc) return rc;
     }
     if (u_curr) {
         rc = r->prec == 32 ? field_in_t<float>(r, u_curr, (float *)r->u[r->cur])
                            : field_in_t<double>(r, u_curr, (double *)r->u[r->cur]);
+        if (rc) return rc;
+        rc = gather_ub_slot(r, r->cur, r->cur ^ 1);  // slot cur^1 = u^n (read by the next step)
         if (rc) return rc;
     }
     const size_t n = (size_t)r->nb * r->MB * r->s;

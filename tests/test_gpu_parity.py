@@ -166,6 +166,39 @@ def test_fd_mm_random_state(orc, precision, MB):
     assert abs(eo - eg) <= 1e-9 * abs(eo)
 
 
+@pytest.mark.parametrize("precision,MB", [(32, 0), (32, 3), (64, 2)])
+def test_source_on_boundary_node_and_split_set_state(orc, precision, MB):
+    """The source on a wall voxel (a boundary node, 0 < K < 6): the node's
+    two-slot u_b ring must follow the source injection; the state is set in
+    two calls (u^{n-1} only, then u^n only), each refreshing one ring slot."""
+    mask = I.lshape_mask(40, 34, 22).numpy()
+    mm = I.material_map(torch.from_numpy(mask), "random", 4).numpy()
+    if MB:
+        beta0, D, E, F = I.fd_tables(4, MB, seed=7)
+    else:
+        beta0, D, E, F = np.array([0.05, 0.2, 0.6, 0.9]), None, None, None
+    o, g = pair(orc, mask, precision, beta0, D, E, F, matmap=mm)
+    K = o.classification()[0]
+    walls = np.argwhere((K > 0) & (K < 6))
+    z, y, x = walls[len(walls) // 3]
+    dt = np.float32 if precision == 32 else np.float64
+    rng = np.random.default_rng(11)
+    up = rng.uniform(-1, 1, mask.shape).astype(dt)
+    uc = rng.uniform(-1, 1, mask.shape).astype(dt)
+    o.set_state(up, uc)
+    g.set_state(u_prev=up)
+    g.set_state(u_curr=uc)
+    for r in (o, g):
+        r.set_source((int(x), int(y), int(z)), I.gaussian_pulse(80, 6.0))
+        r.set_receivers([(int(x), int(y), int(z))])
+        r.step(150)
+    assert_close(o.read_receivers(), g.read_receivers(), precision, "receiver at the source")
+    co, po = o.read_field()
+    cg, pg = g.read_field()
+    assert_close(co, cg, precision, "u^n")
+    assert_close(po, pg, precision, "u^{n-1}")
+
+
 def test_graph_and_direct_launches_agree(orc):
     """CUDA-graph replay (steps in blocks of 16) and one-by-one launches with
     profiling give identical bits."""
