@@ -206,6 +206,9 @@ def run_rafd(args, rank, world, local_rank):
                      z_begin=z0, z_end=z1, mask_z0=mz0, dims=(nx, ny, nz))
     if world > 1 and args.transport == "ipc":
         connect_ipc(room, rank, world)
+    tb = args.tb if world == 1 else 1  # temporal blocking: whole rooms on one GPU
+    if tb == 2:
+        room.set_temporal_blocking(2)
     t_create = time.perf_counter() - t_c
     del mask, mm
     torch.cuda.empty_cache()
@@ -241,6 +244,7 @@ def run_rafd(args, rank, world, local_rank):
     room.set_profiling(False)
     rec = room.read_receivers()
 
+    info = room.get_info()
     t = torch.tensor([ms, float(info["n_inside"]), float(info["bytes_per_step"]), float(launches),
                       kt["volume_ms"], kt["boundary_ms"], kt["other_ms"]], dtype=torch.float64,
                      device=dev)
@@ -264,7 +268,12 @@ def run_rafd(args, rank, world, local_rank):
         bnd_ms = kt["boundary_ms"] / args.steps if kt["boundary_launches"] else 0.0
         # the fused kernel moves the whole step's algorithmic bytes (volume + boundary)
         vol_bytes = info["bytes_per_step"] if fused else info["volume_bytes"]
-        vol_gbs = vol_bytes / (vol_ms * 1e-3) / 1e9
+        n_mask = info["n_mask"]
+        if tb == 2:
+            # k_volume2 per launch (two steps): reads u^{n-1}, u^n, K, writes u^{n+1}, u^{n+2}
+            vol_bytes = n_mask * 1 + info["n_inside"] * 4 * (prec // 8)
+        launch_ms = kt["volume_ms"] / max(1, kt["volume_launches"])
+        vol_gbs = vol_bytes / (launch_ms * 1e-3) / 1e9
         bnd_gbs = info["boundary_bytes"] / (bnd_ms * 1e-3) / 1e9 if (info["n_boundary"] and bnd_ms > 0) else None
         step_gbs = bytes_total * args.steps / (ms_max * 1e-3) / 1e9 / world
         traffic = None
@@ -290,21 +299,28 @@ def run_rafd(args, rank, world, local_rank):
                 "n_boundary_rank0": info["n_boundary"], "parallelism": f"z-slab x{world}",
                 "l2": "inputs larger than L2 (working set %.1f GB/GPU vs 126 MB L2)" % (info["device_bytes"] / 1e9),
                 "timed": "profiled launches (CUDA events around every kernel) on the room stream",
+                "steps_per_sweep": tb,
             },
             "roofline": {
-                "bound": "hbm", "kernel": "k_volume_tma (volume + fused FD-MM boundary)" if fused else "k_volume_tma",
+                "bound": "hbm",
+                "kernel": "k_volume2 (two leapfrog steps per sweep)" if tb == 2 else
+                          ("k_volume_tma (volume + fused FD-MM boundary)" if fused else "k_volume_tma"),
                 "achieved": round(vol_gbs, 1), "peak": peak,
                 "unit": "GB/s", "frac": round(vol_gbs / peak, 4), "traffic": traffic,
                 "algorithmic_bytes_per_launch": vol_bytes,
-                "avg_launch_ms": round(vol_ms, 5), "launches_per_step": kt["volume_launches"] // args.steps,
+                "avg_launch_ms": round(launch_ms, 5), "launches_per_step": kt["volume_launches"] / args.steps,
                 "peak_source": peak_src,
             },
             "kernels": {
                 "volume_ms_per_step": round(vol_ms, 5), "boundary_ms_per_step": round(bnd_ms, 5),
                 "other_ms_per_step": round(kt["other_ms"] / args.steps, 5),
+                "shell_ms_per_step": round(kt["shell_ms"] / args.steps, 5),
+                "n_shell": info["n_shell"],
                 "boundary_gbs": None if bnd_gbs is None else round(bnd_gbs, 1),
                 "boundary_share": round(bnd_ms / (ms_max / args.steps), 4),
                 "fused_boundary": fused,
+                # the one-step-per-sweep method's algorithmic bytes (SURVEY §8(d) B_step) per
+                # step over the measured time: > 1 means temporal blocking beats that roofline
                 "step_algorithmic_gbs_per_gpu": round(step_gbs, 1),
                 "step_frac_of_peak": round(step_gbs / peak, 4),
             },
@@ -361,11 +377,17 @@ def run_e2e(args, cfg, prec, beta0, D, E, F, rank, world, local_rank, plan, mult
         connect_ipc(room, rank, world)
     room.set_source(I.source_position((nx, ny, nz), mask_np), sig)
     room.set_receivers(rcv)
+    tb = args.tb if world == 1 else 1
+    if tb == 2:
+        room.set_temporal_blocking(2)
     d2h = 0
-    for _ in range(steps):
-        room.step(1)
-        r = room.read_receivers(cap=1)
+    done = 0
+    while done < steps:
+        k = min(tb, steps - done)  # a double step with temporal blocking: read both samples
+        room.step(k)
+        r = room.read_receivers(cap=k)
         d2h += r.shape[0] * r.shape[1] * (prec // 8)
+        done += k
     room.synchronize()
     t1 = time.perf_counter()
     n_in = room.get_info()["n_inside"]
@@ -382,7 +404,8 @@ def run_e2e(args, cfg, prec, beta0, D, E, F, rank, world, local_rank, plan, mult
             "h2d_bytes_per_step": int(h2d // steps), "d2h_bytes_per_step": int(d2h // steps),
             "wall_s": round(tmax, 3),
             "includes": "rafd_create from pinned host mask+matmap (H2D, device classification), "
-                        "set_source/set_receivers, per step rafd_step(1)+rafd_read_receivers (D2H), destroy"}
+                        "set_source/set_receivers, per step rafd_step(1)+rafd_read_receivers (D2H), destroy"
+                        + ("; temporal blocking: rafd_step(2) + a read of both samples per call" if tb == 2 else "")}
 
 
 def oracle_sample(cfg, nplanes):
@@ -452,6 +475,8 @@ def main():
     ap.add_argument("--config", default="C4")
     ap.add_argument("--precision", type=int, default=None)
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--tb", type=int, default=2, choices=[1, 2],
+                    help="steps per HBM sweep (temporal blocking; whole rooms on one GPU only)")
     ap.add_argument("--transport", default="nccl", choices=["nccl", "ipc"],
                     help="halo exchange for --gpus > 1: NCCL send/recv, or CUDA-IPC peer copies "
                          "ordered by GPU-side stream waits (rafd_ipc_connect)")

@@ -121,6 +121,9 @@ typedef struct rafd_info {
     int32_t pitch;           /* padded x pitch in elements                              */
     int32_t fused;           /* 1: the boundary update runs inside the volume kernel     */
     int32_t scheme;          /* RAFD_SCHEME_*                                          */
+    int32_t steps_per_sweep; /* 1, or 2 with temporal blocking (rafd_set_temporal_blocking) */
+    int32_t reserved_;
+    int64_t n_shell;         /* voxels recomputed after the boundary update (temporal blocking) */
 } rafd_info;
 
 /* Per-kernel device times accumulated while profiling is on (CUDA events on
@@ -129,6 +132,8 @@ typedef struct rafd_info {
 typedef struct rafd_kernel_times {
     double volume_ms, boundary_ms, other_ms;
     int64_t volume_launches, boundary_launches, other_launches;
+    double shell_ms;         /* the shell recompute of temporal blocking */
+    int64_t shell_launches;
 } rafd_kernel_times;
 
 /* Create a room: validates lambda / tables / dims, copies mask and matmap to
@@ -169,6 +174,21 @@ int rafd_set_step(rafd_room *r, int64_t n);
 /* Enqueue nsteps time steps (volume kernel, boundary kernel, source,
  * receivers, rotation).  Asynchronous w.r.t. the host. */
 int rafd_step(rafd_room *r, int64_t nsteps);
+
+/* Temporal blocking: steps_per_sweep = 2 makes
+ * rafd_step advance two leapfrog steps per pass over the grid.  The volume
+ * update of Listing 2 for step n+2 reads only u^{n+1} on a
+ * voxel's 7-point star, so one z-march computes u^{n+1} and, one plane behind,
+ * u^{n+2}; the boundary update of step n+1 (Listings 3/4, PAPER.md:371-377,
+ * 415-440) and the source then run, and the voxels whose star holds a boundary
+ * node or the source (the "shell") get their u^{n+2} recomputed before the
+ * boundary update of step n+2.  Results are bitwise those of single steps
+ * (same expressions, same order).  Allocates a second pair of field buffers
+ * (the two steps are written out of place) and the shell list; an odd step
+ * count ends with one single step.  1 switches back (buffers are kept).
+ * Errors: INVAL (not 1 or 2), STATE (a z slab, a fused or single-kernel
+ * scheme, or the v0 kernel), NOMEM, CUDA. */
+int rafd_set_temporal_blocking(rafd_room *r, int32_t steps_per_sweep);
 
 /* Step the n slabs of one room held by this process (created with nranks = n,
  * rank = k, nccl_id = NULL, consecutive [z_begin, z_end)), on one or several

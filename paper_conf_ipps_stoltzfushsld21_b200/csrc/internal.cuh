@@ -62,8 +62,8 @@ template <typename T> struct Ctl {
 };
 
 struct KernelTimes {
-    double volume_ms = 0, boundary_ms = 0, other_ms = 0;
-    int64_t volume_n = 0, boundary_n = 0, other_n = 0;
+    double volume_ms = 0, boundary_ms = 0, other_ms = 0, shell_ms = 0;
+    int64_t volume_n = 0, boundary_n = 0, other_n = 0, shell_n = 0;
 };
 
 // ------------------------------------------------------------------ launchers
@@ -95,8 +95,22 @@ cudaError_t volume_plan_fuse(void *plan, const Grid &g, const uint8_t *K, int64_
 bool volume_plan_fused(const void *plan);
 cudaError_t volume_plan_occupancy(void *plan, const Grid &g, const uint8_t *K, cudaStream_t s);
 template <typename T>
-cudaError_t volume_plan_create(const Grid &g, void *u0, void *u1, uint8_t *K, int nsm, void **plan);
+cudaError_t volume_plan_create(const Grid &g, void *const u[4], uint8_t *K, int nsm, void **plan);
 void volume_plan_destroy(void *plan);
+// temporal blocking (twostep.cu): the two-step volume kernel over the four
+// field buffers (cur_buf = u^n, prev_buf = u^{n-1} -> out1 = u^{n+1}, out2 =
+// u^{n+2}) and the shell recompute of u^{n+2} (list built by the plan)
+template <typename T>
+cudaError_t twostep_plan_create(const Grid &g, void *const u[4], uint8_t *K_alloc, const uint8_t *K, bool idx64,
+                                int nsm, cudaStream_t s, void **plan, int64_t *n_shell);
+void twostep_plan_destroy(void *plan);
+cudaError_t twostep_set_source(void *plan, int64_t pos, const Grid &g);
+template <typename T>
+cudaError_t launch_volume2(const void *plan, const Grid &g, int cur_buf, int prev_buf, T *out1, T *out2,
+                           double lambda, cudaStream_t s);
+template <typename T>
+cudaError_t launch_shell(const void *plan, const Grid &g, const T *u1, const T *u0, const uint8_t *K, T *out,
+                         double lambda, cudaStream_t s);
 template <typename T>
 cudaError_t launch_boundary(int MB, bool idx64, const void *bpos, const uint8_t *Kb,
                             const uint8_t *matb, int64_t i_lo, int64_t i_hi, int64_t Nb, T *unext,

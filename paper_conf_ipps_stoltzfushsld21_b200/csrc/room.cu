@@ -90,8 +90,17 @@ struct rafd_room {
     double lambda = 0;
     Grid g{};
     int nsm = 148;
-    void *u[2] = {nullptr, nullptr};
-    int cur = 0;  // u[cur] = u^n
+    // field buffers: two pairs.  u[pair + cur] = u^n, u[pair + (cur^1)] =
+    // u^{n-1}; a single step writes u^{n+1} in place over u^{n-1} (cur ^= 1), a
+    // double step of the two-step kernel (twostep.cu) writes the other pair
+    // (pair ^= 2, cur unchanged).  The second pair exists only with temporal
+    // blocking on (rafd_set_temporal_blocking).
+    void *u[4] = {nullptr, nullptr, nullptr, nullptr};
+    int cur = 0;
+    int pair = 0;
+    int tb = 1;              // steps per HBM sweep (1 or 2)
+    void *tbplan = nullptr;  // two-step kernel maps + shell list
+    int64_t n_shell = 0;
     uint8_t *K = nullptr, *K_alloc = nullptr;
     int64_t nb = 0;
     bool idx64 = false;
@@ -116,7 +125,7 @@ struct rafd_room {
     int64_t launches = 0;
     // CUDA graphs of G steps, one per starting parity
     static const int G = 16;
-    cudaGraphExec_t graph[2] = {nullptr, nullptr};
+    cudaGraphExec_t graph[4] = {nullptr, nullptr, nullptr, nullptr};  // index pair + cur
     int graph_kernels = 0;
     // profiling
     bool profiling = false;
@@ -412,7 +421,7 @@ template <typename T> static int create_t(rafd_room *r, const rafd_room_desc *d)
     CK(cudaMemcpy(r->ctl, &c, sizeof c, cudaMemcpyHostToDevice));
     const char *env = getenv("RAFD_VOLUME_KERNEL");
     if (!(env && strcmp(env, "v0") == 0)) {
-        CK(volume_plan_create<T>(g, r->u[0], r->u[1], r->K_alloc, r->nsm, &r->vplan));
+        CK(volume_plan_create<T>(g, r->u, r->K_alloc, r->nsm, &r->vplan));
         const char *sk = getenv("RAFD_SKIP_EMPTY");  // skipping of all-outside tile-planes (default on)
         if (!(sk && strcmp(sk, "0") == 0)) CK(volume_plan_occupancy(r->vplan, g, r->K, r->stream));
     }
@@ -499,7 +508,7 @@ extern "C" int rafd_create(const rafd_room_desc *d, rafd_room **out)
 
 static void free_graphs(rafd_room *r)
 {
-    for (int p = 0; p < 2; p++)
+    for (int p = 0; p < 4; p++)
         if (r->graph[p]) {
             cudaGraphExecDestroy(r->graph[p]);
             r->graph[p] = nullptr;
@@ -519,7 +528,8 @@ extern "C" void rafd_destroy(rafd_room *r)
     if (r->ev_halo) cudaEventDestroy(r->ev_halo);
     if (r->comm_stream) cudaStreamDestroy(r->comm_stream);
     if (r->vplan) volume_plan_destroy(r->vplan);
-    void *ps[] = {r->u[0], r->u[1], r->K_alloc, r->bpos, r->bidx, r->Kb, r->matb, r->ub, r->gst, r->vst,
+    if (r->tbplan) twostep_plan_destroy(r->tbplan);
+    void *ps[] = {r->u[0], r->u[1], r->u[2], r->u[3], r->K_alloc, r->bpos, r->bidx, r->Kb, r->matb, r->ub, r->gst, r->vst,
                   r->tab, r->DF, r->ctl, r->sig, r->rcv_pos, r->rec};
     for (void *p : ps)
         if (p) cudaFree(p);
@@ -602,6 +612,8 @@ static int set_source_t(rafd_room *r, int32_t x, int32_t y, int32_t z, const dou
         }
         r->src_z = z;
     }
+    // temporal blocking: the source's 7-point star is recomputed with the shell
+    if (r->tbplan) CK(twostep_set_source(r->tbplan, c.src_pos, r->g));
     return push_ctl<T>(r, c);
 }
 
@@ -682,32 +694,37 @@ template <typename T> static int ensure_rec(rafd_room *r, int64_t more)
 }
 
 // ------------------------------------------------------------------ stepping
-template <typename T> static cudaError_t enqueue_step(rafd_room *r, int cur, cudaStream_t s, bool prof)
+// the profiling wrapper: CUDA events around one launch on stream s
+template <typename Fn> static cudaError_t timed_launch(rafd_room *r, cudaStream_t s, bool prof, int kind, Fn fn)
+{
+    if (!prof) return fn();
+    cudaEvent_t a, b;
+    if (r->ev_pool.size() >= 2) {
+        a = r->ev_pool.back();
+        r->ev_pool.pop_back();
+        b = r->ev_pool.back();
+        r->ev_pool.pop_back();
+    } else {
+        cudaEventCreate(&a);
+        cudaEventCreate(&b);
+    }
+    cudaEventRecord(a, s);
+    cudaError_t e = fn();
+    cudaEventRecord(b, s);
+    r->evs.push_back({kind, a, b});
+    return e;
+}
+
+// one step from the state (pair, cur): u^n = u[pair+cur] -> u^{n+1} in place over u[pair+(cur^1)]
+template <typename T> static cudaError_t enqueue_step(rafd_room *r, int pair, int cur, cudaStream_t s, bool prof)
 {
     const Grid &g = r->g;
-    T *uc = (T *)r->u[cur];
-    T *un = (T *)r->u[cur ^ 1];
-    auto timed = [&](int kind, auto fn) -> cudaError_t {
-        if (!prof) return fn();
-        cudaEvent_t a, b;
-        if (r->ev_pool.size() >= 2) {
-            a = r->ev_pool.back();
-            r->ev_pool.pop_back();
-            b = r->ev_pool.back();
-            r->ev_pool.pop_back();
-        } else {
-            cudaEventCreate(&a);
-            cudaEventCreate(&b);
-        }
-        cudaEventRecord(a, s);
-        cudaError_t e = fn();
-        cudaEventRecord(b, s);
-        r->evs.push_back({kind, a, b});
-        return e;
-    };
+    T *uc = (T *)r->u[pair + cur];
+    T *un = (T *)r->u[pair + (cur ^ 1)];
+    auto timed = [&](int kind, auto fn) -> cudaError_t { return timed_launch(r, s, prof, kind, fn); };
     const FusedArgs<T> fa = fused_args<T>(r);
     cudaError_t e = timed(0, [&] {
-        return launch_volume<T>(g, uc, un, r->K, r->lambda, 0, g.lnz, s, r->vplan, cur,
+        return launch_volume<T>(g, uc, un, r->K, r->lambda, 0, g.lnz, s, r->vplan, pair + cur,
                                 (r->fused || r->scheme) ? &fa : nullptr);
     });
     if (e != cudaSuccess) return e;
@@ -722,6 +739,33 @@ template <typename T> static cudaError_t enqueue_step(rafd_room *r, int cur, cud
     e = timed(2, [&] { return launch_src_rcv<T>(un, ub_slot<T>(r, cur), ctl_of<T>(r), s); });
     if (e != cudaSuccess) return e;
     return cudaSuccess;
+}
+
+// one double step of the two-step kernel (twostep.cu) from the state (pair,
+// cur): A = u^{n-1}, B = u^n -> C = u^{n+1}, D = u^{n+2} in the other pair,
+// placed so that the state after it is (pair^2, cur).  The u_b slots follow
+// the steps (slot cur for step n+1, cur^1 for step n+2), as two single steps.
+template <typename T> static cudaError_t enqueue_step2(rafd_room *r, int pair, int cur, cudaStream_t s, bool prof)
+{
+    const Grid &g = r->g;
+    const int bA = pair + (cur ^ 1), bB = pair + cur, bC = (pair ^ 2) + (cur ^ 1), bD = (pair ^ 2) + cur;
+    T *B = (T *)r->u[bB], *C = (T *)r->u[bC], *D = (T *)r->u[bD];
+    auto bnd = [&](T *un, int slot) -> cudaError_t {
+        if (r->nb == 0) return cudaSuccess;
+        return timed_launch(r, s, prof, 1, [&] {
+            return launch_boundary<T>(r->MB, r->idx64, r->bpos, r->Kb, r->matb, 0, r->nb, r->nb, un,
+                                      ub_slot<T>(r, slot), (T *)r->gst, (T *)r->vst, (const T *)r->tab, r->M,
+                                      r->lambda, s);
+        });
+    };
+    cudaError_t e = timed_launch(r, s, prof, 0, [&] { return launch_volume2<T>(r->tbplan, g, bB, bA, C, D, r->lambda, s); });
+    if (e == cudaSuccess) e = bnd(C, cur);
+    if (e == cudaSuccess) e = timed_launch(r, s, prof, 2, [&] { return launch_src_rcv<T>(C, ub_slot<T>(r, cur), ctl_of<T>(r), s); });
+    if (e == cudaSuccess)
+        e = timed_launch(r, s, prof, 3, [&] { return launch_shell<T>(r->tbplan, g, C, B, r->K, D, r->lambda, s); });
+    if (e == cudaSuccess) e = bnd(D, cur ^ 1);
+    if (e == cudaSuccess) e = timed_launch(r, s, prof, 2, [&] { return launch_src_rcv<T>(D, ub_slot<T>(r, cur ^ 1), ctl_of<T>(r), s); });
+    return e;
 }
 
 // ---- slab step, edge planes first: phase 0 = the first and
@@ -825,18 +869,27 @@ template <typename T> static cudaError_t enqueue_step_nccl(rafd_room *r, bool pr
 }
 
 static int kernels_per_step(const rafd_room *r) { return 2 + (r->nb > 0 && !r->fused && !r->scheme ? 1 : 0); }
+static int kernels_per_double_step(const rafd_room *r) { return 4 + (r->nb > 0 ? 2 : 0); }
 
-template <typename T> static int build_graph(rafd_room *r, int parity)
+// a graph of G steps from the state (pair, cur) (index pair + cur); it ends in
+// the same state (G single steps flip cur an even number of times, G/2 double
+// steps flip pair an even number of times)
+template <typename T> static int build_graph(rafd_room *r, int pair, int cur)
 {
     cudaGraph_t gr;
     CK(cudaStreamBeginCapture(r->cap_stream, cudaStreamCaptureModeThreadLocal));
     cudaError_t e = cudaSuccess;
-    for (int k = 0; k < rafd_room::G && e == cudaSuccess; k++)
-        e = enqueue_step<T>(r, parity ^ (k & 1), r->cap_stream, false);
+    if (r->tb == 2) {
+        for (int k = 0; k < rafd_room::G / 2 && e == cudaSuccess; k++)
+            e = enqueue_step2<T>(r, pair ^ (2 * (k & 1)), cur, r->cap_stream, false);
+    } else {
+        for (int k = 0; k < rafd_room::G && e == cudaSuccess; k++)
+            e = enqueue_step<T>(r, pair, cur ^ (k & 1), r->cap_stream, false);
+    }
     cudaError_t e2 = cudaStreamEndCapture(r->cap_stream, &gr);
     if (e != cudaSuccess) return set_err(RAFD_E_CUDA, "capture: %s", cudaGetErrorString(e));
     CK(e2);
-    CK(cudaGraphInstantiate(&r->graph[parity], gr, 0));
+    CK(cudaGraphInstantiate(&r->graph[pair + cur], gr, 0));
     cudaGraphDestroy(gr);
     return RAFD_OK;
 }
@@ -848,11 +901,20 @@ template <typename T> static int step_t(rafd_room *r, int64_t nsteps)
     const int kps = kernels_per_step(r);
     int64_t done = 0;
     const bool use_graph = !r->profiling && !r->halo && !r->ipc && nsteps >= rafd_room::G;
+    const int gi = r->pair + r->cur;
     while (use_graph && nsteps - done >= rafd_room::G) {
-        if (!r->graph[r->cur] && (rc = build_graph<T>(r, r->cur))) return rc;
-        CK(cudaGraphLaunch(r->graph[r->cur], r->stream));
-        done += rafd_room::G;  // G is even: parity unchanged
-        r->launches += (int64_t)kps * rafd_room::G;
+        if (!r->graph[gi] && (rc = build_graph<T>(r, r->pair, r->cur))) return rc;
+        CK(cudaGraphLaunch(r->graph[gi], r->stream));
+        done += rafd_room::G;  // G is even: state unchanged
+        r->launches += r->tb == 2 ? (int64_t)kernels_per_double_step(r) * (rafd_room::G / 2) : (int64_t)kps * rafd_room::G;
+    }
+    // temporal blocking: double steps, an odd last step runs single
+    while (r->tb == 2 && nsteps - done >= 2) {
+        cudaError_t e = enqueue_step2<T>(r, r->pair, r->cur, r->stream, r->profiling);
+        if (e != cudaSuccess) return set_err(RAFD_E_CUDA, "step: %s", cudaGetErrorString(e));
+        r->launches += kernels_per_double_step(r);
+        r->pair ^= 2;
+        done += 2;
     }
     for (; done < nsteps; done++) {
         cudaError_t e;
@@ -865,7 +927,7 @@ template <typename T> static int step_t(rafd_room *r, int64_t nsteps)
             if (e == cudaErrorUnknown) return set_err(RAFD_E_CUDA, "%s", halo_last_error());
             r->launches += kernels_per_phase(r, 0) + kernels_per_phase(r, 1);
         } else {
-            e = enqueue_step<T>(r, r->cur, r->stream, r->profiling);
+            e = enqueue_step<T>(r, r->pair, r->cur, r->stream, r->profiling);
             r->launches += kps;
         }
         if (e != cudaSuccess) return set_err(RAFD_E_CUDA, "step: %s", cudaGetErrorString(e));
@@ -1088,10 +1150,11 @@ extern "C" int rafd_read_field(rafd_room *r, void *u_curr, void *u_prev)
     if (!r) return set_err(RAFD_E_INVAL, "null room");
     CK(cudaSetDevice(r->device));
     int rc = RAFD_OK;
-    if (u_curr) rc = r->prec == 32 ? field_out_t<float>(r, (const float *)r->u[r->cur], u_curr)
-                                   : field_out_t<double>(r, (const double *)r->u[r->cur], u_curr);
-    if (!rc && u_prev) rc = r->prec == 32 ? field_out_t<float>(r, (const float *)r->u[r->cur ^ 1], u_prev)
-                                          : field_out_t<double>(r, (const double *)r->u[r->cur ^ 1], u_prev);
+    const int bc = r->pair + r->cur, bp = r->pair + (r->cur ^ 1);
+    if (u_curr) rc = r->prec == 32 ? field_out_t<float>(r, (const float *)r->u[bc], u_curr)
+                                   : field_out_t<double>(r, (const double *)r->u[bc], u_curr);
+    if (!rc && u_prev) rc = r->prec == 32 ? field_out_t<float>(r, (const float *)r->u[bp], u_prev)
+                                          : field_out_t<double>(r, (const double *)r->u[bp], u_prev);
     return rc;
 }
 
@@ -1184,19 +1247,20 @@ extern "C" int rafd_set_state(rafd_room *r, const void *u_prev, const void *u_cu
     CK(cudaSetDevice(r->device));
     CK(cudaStreamSynchronize(r->stream));
     int rc = RAFD_OK;
+    const int bc = r->pair + r->cur, bp = r->pair + (r->cur ^ 1);
     if (u_prev) {
-        rc = r->prec == 32 ? field_in_t<float>(r, u_prev, (float *)r->u[r->cur ^ 1])
-                           : field_in_t<double>(r, u_prev, (double *)r->u[r->cur ^ 1]);
+        rc = r->prec == 32 ? field_in_t<float>(r, u_prev, (float *)r->u[bp])
+                           : field_in_t<double>(r, u_prev, (double *)r->u[bp]);
         if (rc) return rc;
         // u_b slot cur = u^{n-1} at the boundary nodes (reading R8)
-        rc = gather_ub_slot(r, r->cur ^ 1, r->cur);
+        rc = gather_ub_slot(r, bp, r->cur);
         if (rc) return rc;
     }
     if (u_curr) {
-        rc = r->prec == 32 ? field_in_t<float>(r, u_curr, (float *)r->u[r->cur])
-                           : field_in_t<double>(r, u_curr, (double *)r->u[r->cur]);
+        rc = r->prec == 32 ? field_in_t<float>(r, u_curr, (float *)r->u[bc])
+                           : field_in_t<double>(r, u_curr, (double *)r->u[bc]);
         if (rc) return rc;
-        rc = gather_ub_slot(r, r->cur, r->cur ^ 1);  // slot cur^1 = u^n (read by the next step)
+        rc = gather_ub_slot(r, bc, r->cur ^ 1);  // slot cur^1 = u^n (read by the next step)
         if (rc) return rc;
     }
     const size_t n = (size_t)r->nb * r->MB * r->s;
@@ -1238,6 +1302,8 @@ extern "C" int rafd_get_info(rafd_room *r, rafd_info *info)
     info->pitch = (int32_t)r->g.pitch;
     info->fused = r->fused ? 1 : 0;
     info->scheme = r->scheme;
+    info->steps_per_sweep = r->tb;
+    info->n_shell = r->n_shell;
     return RAFD_OK;
 }
 
@@ -1248,7 +1314,7 @@ extern "C" int rafd_energy(rafd_room *r, double *H)
     double *acc = nullptr;
     CK(cudaMalloc((void **)&acc, 3 * sizeof(double)));
     CK(cudaMemsetAsync(acc, 0, 3 * sizeof(double), r->stream));
-    const void *un1 = r->u[r->cur], *un = r->u[r->cur ^ 1];
+    const void *un1 = r->u[r->pair + r->cur], *un = r->u[r->pair + (r->cur ^ 1)];
     cudaError_t e;
     if (r->prec == 32) {
         e = launch_energy<float>(r->g, (const float *)un1, (const float *)un, r->K, acc, r->stream);
@@ -1279,6 +1345,9 @@ static void resolve_events(rafd_room *r)
         } else if (e.kind == 1) {
             r->kt.boundary_ms += ms;
             r->kt.boundary_n++;
+        } else if (e.kind == 3) {
+            r->kt.shell_ms += ms;
+            r->kt.shell_n++;
         } else {
             r->kt.other_ms += ms;
             r->kt.other_n++;
@@ -1310,10 +1379,60 @@ extern "C" int rafd_get_kernel_times(rafd_room *r, rafd_kernel_times *t)
     t->volume_launches = r->kt.volume_n;
     t->boundary_launches = r->kt.boundary_n;
     t->other_launches = r->kt.other_n;
+    t->shell_ms = r->kt.shell_ms;
+    t->shell_launches = r->kt.shell_n;
     return RAFD_OK;
 }
 
 extern "C" int64_t rafd_launch_count(rafd_room *r) { return r ? r->launches : 0; }
+
+// ------------------------------------------------------------------ temporal blocking
+template <typename T> static int enable_twostep_t(rafd_room *r)
+{
+    int rc;
+    const size_t fb = (size_t)r->g.total * sizeof(T) + 64;
+    for (int k = 2; k < 4; k++)
+        if (!r->u[k]) {
+            if ((rc = dmalloc(r, &r->u[k], fb))) return rc;
+            CK(cudaMemsetAsync(r->u[k], 0, fb, r->stream));
+        }
+    if (!r->tbplan) {
+        // the single-step kernel needs TMA maps of the second pair too
+        volume_plan_destroy(r->vplan);
+        r->vplan = nullptr;
+        CK(volume_plan_create<T>(r->g, r->u, r->K_alloc, r->nsm, &r->vplan));
+        const char *sk = getenv("RAFD_SKIP_EMPTY");
+        if (!(sk && strcmp(sk, "0") == 0)) CK(volume_plan_occupancy(r->vplan, r->g, r->K, r->stream));
+        CK(twostep_plan_create<T>(r->g, r->u, r->K_alloc, r->K, r->idx64, r->nsm, r->stream, &r->tbplan, &r->n_shell));
+        r->device_bytes += r->n_shell * (r->idx64 ? 8 : 4) + 56;
+        Ctl<T> c;
+        if ((rc = pull_ctl<T>(r, c))) return rc;
+        CK(twostep_set_source(r->tbplan, c.src_pos, r->g));
+    }
+    CK(cudaStreamSynchronize(r->stream));
+    return RAFD_OK;
+}
+
+extern "C" int rafd_set_temporal_blocking(rafd_room *r, int32_t steps_per_sweep)
+{
+    if (!r || (steps_per_sweep != 1 && steps_per_sweep != 2))
+        return set_err(RAFD_E_INVAL, "steps_per_sweep must be 1 or 2");
+    CK(cudaSetDevice(r->device));
+    if (steps_per_sweep == r->tb) return RAFD_OK;
+    CK(cudaStreamSynchronize(r->stream));
+    if (steps_per_sweep == 2) {
+        if (r->nranks > 1 || r->halo || r->ipc || r->local_slab)
+            return set_err(RAFD_E_STATE, "temporal blocking needs a whole room on one GPU (not a z slab)");
+        if (r->scheme != 0 || r->fused)
+            return set_err(RAFD_E_STATE, "temporal blocking runs the two-kernel scheme (not fused, not Listing 1/6)");
+        if (!r->vplan) return set_err(RAFD_E_STATE, "temporal blocking needs the TMA volume kernel (not v0)");
+        int rc = r->prec == 32 ? enable_twostep_t<float>(r) : enable_twostep_t<double>(r);
+        if (rc) return rc;
+    }
+    free_graphs(r);  // the step sequence changed
+    r->tb = steps_per_sweep;
+    return RAFD_OK;
+}
 
 // ------------------------------------------------------------------ host-only helpers
 extern "C" int rafd_slab_plan(int32_t nx, int32_t ny, int32_t nz, const uint8_t *mask, int32_t precision,

@@ -1,0 +1,596 @@
+// twostep.cu -- temporal blocking: two leapfrog steps per HBM sweep (SURVEY
+// §8(f) row f4).
+//
+// The volume update (Listing 2 kernel 1) of step n+1 at a
+// voxel needs u^n on its 7-point star; that of step n+2 needs u^{n+1} there.
+// One z-march can therefore produce both levels: the CTA computes u^{n+1} of
+// plane q (kept in shared memory and registers) and, one plane behind, u^{n+2}
+// of plane q-1 from it.  Per voxel and double step it reads u^{n-1}, u^n, K and
+// writes u^{n+1}, u^{n+2}: 4s+1 bytes for two steps instead of 2(3s+1).
+//
+// Three things make this exact (bitwise equal to two single steps):
+//  * out of place: u^{n-1}, u^n are read from one buffer pair and u^{n+1},
+//    u^{n+2} written to the other (four field buffers), so overlapping tiles
+//    never read a value another CTA has already advanced;
+//  * overlapped tiles: the u^{n+1} a tile's step n+2 needs from its x/y
+//    neighbours is recomputed (step n+1 runs on the tile plus one ring of
+//    voxels; 30 of the 32 lane vectors, TY of the TY+2 rows are stored);
+//  * the "shell": a voxel's u^{n+2} from this kernel is final only if neither
+//    the voxel nor a face neighbour is a boundary node (their u^{n+1} changes
+//    in the boundary kernel, rows a3/a4) or the source voxel (row a5).  Those
+//    voxels (a list built once per room; the source and its neighbours in a
+//    7-entry side list) are recomputed by k_shell after the boundary kernel
+//    and the source injection of step n+1, with the same arithmetic.
+//
+// Sequence of one double step (room.cu, enqueue_step2):
+//   k_volume2 (A=u^{n-1}, B=u^n -> C=u^{n+1}, D=u^{n+2} provisional)
+//   k_boundary(C), k_src_rcv(C)          -- step n+1 final
+//   k_shell   (C, B -> D at shell voxels) -- step n+2 volume final
+//   k_boundary(D), k_src_rcv(D)          -- step n+2 final
+#include <cuda.h>
+#include <cudaTypedefs.h>
+
+#include <stdlib.h>
+
+#include "internal.cuh"
+
+namespace rafd {
+
+// ------------------------------------------------------------------ PTX helpers
+namespace tb {
+static __device__ __forceinline__ uint32_t smem_u32(const void *p) { return (uint32_t)__cvta_generic_to_shared(p); }
+static __device__ __forceinline__ void mbar_init(uint64_t *b, uint32_t count)
+{
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(b)), "r"(count));
+}
+static __device__ __forceinline__ void mbar_expect_tx(uint64_t *b, uint32_t bytes)
+{
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(b)), "r"(bytes) : "memory");
+}
+static __device__ __forceinline__ void mbar_wait(uint64_t *b, uint32_t parity)
+{
+    asm volatile(
+        "{\n\t.reg .pred p;\n"
+        "WAIT_%=:\n\t"
+        "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n\t"
+        "@!p bra WAIT_%=;\n\t}" ::"r"(smem_u32(b)),
+        "r"(parity)
+        : "memory");
+}
+static __device__ __forceinline__ void tma_load_3d(void *dst, const CUtensorMap *map, uint64_t *bar, int c0, int c1,
+                                                   int c2)
+{
+    asm volatile(
+        "cp.async.bulk.tensor.3d.shared::cluster.global.tile.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3, "
+        "%4}], [%5];" ::"r"(smem_u32(dst)),
+        "l"((uint64_t)map), "r"(c0), "r"(c1), "r"(c2), "r"(smem_u32(bar))
+        : "memory");
+}
+static __device__ __forceinline__ uint64_t policy_evict_first()
+{
+    uint64_t p;
+    asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p));
+    return p;
+}
+static __device__ __forceinline__ void st_v4_hint(void *ptr, uint4 v, uint64_t pol)
+{
+    asm volatile("st.global.L2::cache_hint.v4.b32 [%0], {%1, %2, %3, %4}, %5;" ::"l"(ptr), "r"(v.x), "r"(v.y),
+                 "r"(v.z), "r"(v.w), "l"(pol)
+                 : "memory");
+}
+}  // namespace tb
+
+template <typename T> struct Vec16;
+template <> struct Vec16<float> {
+    static constexpr int N = 4;
+    using K = uint32_t;
+};
+template <> struct Vec16<double> {
+    static constexpr int N = 2;
+    using K = uint16_t;
+};
+
+// Tile geometry.  Step n+1 runs on TX x (TY+2) voxels (32 lanes x one 16-byte
+// vector, rows -1..TY), step n+2 and both stores on the TXO x TY core (lanes
+// 1..30, rows 0..TY-1); u^n is staged with one more ring (a vector in x, a
+// row in y).  SU u^n slots, SP u^{n-1}/K slots, two u^{n+1} planes.
+template <typename T, int TY, int SU, int SP> struct TbGeom {
+    static constexpr int VEC = Vec16<T>::N;
+    static constexpr int TX = 32 * VEC;
+    static constexpr int TXO = TX - 2 * VEC;
+    static constexpr int UROW = TX + 2 * VEC;
+    static constexpr int UR = TY + 4, PR = TY + 2;
+    static constexpr int NW = PR / 2;  // two step-(n+1) rows per warp
+    static constexpr int NT = 32 * NW;
+    static constexpr int U_BYTES = (UR * UROW * (int)sizeof(T) + 127) / 128 * 128;
+    static constexpr int P_BYTES = PR * TX * (int)sizeof(T);
+    // the K box starts at the 16-byte aligned byte at or below the region (TMA
+    // box origins must be 16-byte aligned) and is 16 bytes wider
+    static constexpr int KROW = TX + 16;
+    static constexpr int K_BYTES = (PR * KROW + 127) / 128 * 128;
+    static constexpr int U1_BYTES = PR * TX * (int)sizeof(T);
+    static constexpr int U_TX = UR * UROW * (int)sizeof(T);
+    static constexpr int PK_TX = P_BYTES + PR * KROW;
+    static constexpr int SMEM = SU * U_BYTES + SP * (P_BYTES + K_BYTES) + 2 * U1_BYTES + (SU + SP) * 8 + 128;
+    static_assert(PR % 2 == 0, "TY must be even");
+};
+
+// One 16-byte vector of the volume update (DESIGN.md §4 order): neighbours
+// summed x-1, x+1, y-1, y+1, z-1, z+1; K = 0 keeps `keep` (outside: +0).
+template <typename T>
+static __device__ __forceinline__ void vol_vec(const T *c, const T *ym, const T *yp, const T *zm, const T *zp,
+                                               const T *pv, T left, T right, uint32_t kw, T l2, T *o)
+{
+    using R = rn<T>;
+    constexpr int VEC = Vec16<T>::N;
+#pragma unroll
+    for (int i = 0; i < VEC; i++) {
+        const int nbr = (int)((kw >> (8 * i)) & 0xff);
+        const T xm = i == 0 ? left : c[i - 1];
+        const T xp = i == VEC - 1 ? right : c[i + 1];
+        T s = R::add(xm, xp);
+        s = R::add(s, ym[i]);
+        s = R::add(s, yp[i]);
+        s = R::add(s, zm[i]);
+        s = R::add(s, zp[i]);
+        const T a = R::sub((T)2, R::mul(l2, (T)nbr));
+        T t = R::mul(a, c[i]);
+        t = R::add(t, R::mul(l2, s));
+        o[i] = nbr ? R::sub(t, pv[i]) : pv[i];
+    }
+}
+
+// The two-step kernel.  umap: u^n (box UROW x (TY+4)); pmap: u^{n-1} (TX x
+// (TY+2)); kmap: K (TX x (TY+2)); out1 = u^{n+1}, out2 = u^{n+2} (other pair).
+template <typename T, int TY, int SU, int SP>
+__global__ void __launch_bounds__(TbGeom<T, TY, SU, SP>::NT, 1)
+    k_volume2(const __grid_constant__ CUtensorMap umap, const __grid_constant__ CUtensorMap pmap,
+              const __grid_constant__ CUtensorMap kmap, T *__restrict__ out1, T *__restrict__ out2, Grid g, T l2,
+              int zchunk, int tiles_x, int tiles_y)
+{
+    using G = TbGeom<T, TY, SU, SP>;
+    using KW = typename Vec16<T>::K;
+    constexpr int VEC = G::VEC, TX = G::TX, TXO = G::TXO, UROW = G::UROW;
+    extern __shared__ __align__(128) unsigned char smem_raw[];
+    unsigned char *base = (unsigned char *)(((uintptr_t)smem_raw + 127) & ~(uintptr_t)127);
+    T *us = (T *)base;                                                  // SU u^n slots
+    T *ps = (T *)(base + SU * G::U_BYTES);                              // SP u^{n-1} slots
+    uint8_t *ks = base + SU * G::U_BYTES + SP * G::P_BYTES;             // SP K slots
+    T *u1s = (T *)(base + SU * G::U_BYTES + SP * (G::P_BYTES + G::K_BYTES));  // 2 u^{n+1} planes
+    uint64_t *bar = (uint64_t *)((unsigned char *)u1s + 2 * G::U1_BYTES);
+    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+
+    if (tid == 0) {
+        for (int i = 0; i < SU + SP; i++) tb::mbar_init(&bar[i], 1);
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+    __syncthreads();
+    uint32_t uph = 0, pph = 0;
+    const uint64_t pol = tb::policy_evict_first();
+
+    const int nz = g.lnz;
+    const int nchunks = (nz + zchunk - 1) / zchunk;
+    const int tiles = tiles_x * tiles_y;
+    const int units = nchunks * tiles;
+    // this warp's two step-(n+1) rows, relative to the tile's first core row
+    const int r0 = 2 * warp - 1;
+    for (int unit = blockIdx.x; unit < units; unit += gridDim.x) {
+        const int chunk = unit / tiles, t = unit % tiles;
+        const int ty = t / tiles_x, tx = t % tiles_x;
+        const int pa = 1 + chunk * zchunk;          // first padded plane stored
+        const int pb = min(1 + nz, pa + zchunk);    // one past the last
+        const int ox = tx * TXO, oy = ty * TY;      // core origin (room coordinates)
+        const int ux = g.xo + ox - 2 * VEC;         // u^n box origin (padded x)
+        const int uy = oy - 1;                      // padded row of core row -2
+        const int px = g.xo + ox - VEC, py = oy;    // u^{n-1} box origin (padded)
+        const int kx = px + k_shift(g);              // K bytes of the region start
+        const int kd = kx & 15;                      // its offset in the aligned K box
+        auto issue_u = [&](int p) {
+            const int s = (p + 2) % SU;
+            tb::mbar_expect_tx(&bar[s], G::U_TX);
+            tb::tma_load_3d((unsigned char *)us + s * G::U_BYTES, &umap, &bar[s], ux, uy, p);
+        };
+        auto issue_pk = [&](int p) {
+            const int s = (p + 1) % SP;
+            tb::mbar_expect_tx(&bar[SU + s], G::PK_TX);
+            tb::tma_load_3d((unsigned char *)ps + s * G::P_BYTES, &pmap, &bar[SU + s], px, py, p);
+            tb::tma_load_3d(ks + s * G::K_BYTES, &kmap, &bar[SU + s], kx - kd, py, p);
+        };
+        auto wait_u = [&](int p) {
+            const int s = (p + 2) % SU;
+            tb::mbar_wait(&bar[s], (uph >> s) & 1);
+            uph ^= 1u << s;
+        };
+        auto wait_pk = [&](int p) {
+            const int s = (p + 1) % SP;
+            tb::mbar_wait(&bar[SU + s], (pph >> s) & 1);
+            pph ^= 1u << s;
+        };
+        auto uslot = [&](int p) -> const T * { return us + ((p + 2) % SU) * (G::U_BYTES / (int)sizeof(T)); };
+        // u^n planes pa-2 .. pb+1, u^{n-1}/K planes pa-1 .. pb
+        __syncthreads();  // the previous unit is done with every slot
+        if (tid == 0) {
+            asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+            for (int p = pa - 2; p < pa - 2 + SU && p <= pb + 1; p++) issue_u(p);
+            for (int p = pa - 1; p < pa - 1 + SP && p <= pb; p++) issue_pk(p);
+        }
+        // register windows per row k: u^n at q-1 and q, u^{n+1} at q-2 and q-1, K at q-1
+        T unm[2][VEC], unc[2][VEC], o1m[2][VEC], o1c[2][VEC];
+        KW km[2];
+        wait_u(pa - 2);
+        wait_u(pa - 1);
+        const int col = VEC + lane * VEC;  // this lane's vector in a u^n smem row
+#pragma unroll
+        for (int k = 0; k < 2; k++) {
+            const int sr = r0 + k + 2;  // smem row of step row r in the u^n box
+            *(uint4 *)unm[k] = *(const uint4 *)(uslot(pa - 2) + sr * UROW + col);
+            *(uint4 *)unc[k] = *(const uint4 *)(uslot(pa - 1) + sr * UROW + col);
+#pragma unroll
+            for (int i = 0; i < VEC; i++) o1m[k][i] = o1c[k][i] = (T)0;
+            km[k] = 0;
+        }
+        __syncthreads();  // plane pa-2 lives on in registers only: refill its slot
+        if (tid == 0) {
+            asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+            if (pa - 2 + SU <= pb + 1) issue_u(pa - 2 + SU);
+        }
+        const bool lane_core = lane >= 1 && lane <= 30;
+        const int xv = ox + (lane - 1) * VEC;        // room x of this lane's vector (core lanes)
+        const bool x_ok = lane_core && xv < g.nx;
+        for (int q = pa - 1; q <= pb; q++) {
+            wait_u(q + 1);
+            wait_pk(q);
+            const T *uq = uslot(q), *uqp = uslot(q + 1);
+            const T *pq = ps + ((q + 1) % SP) * (G::P_BYTES / (int)sizeof(T));
+            const uint8_t *kq = ks + ((q + 1) % SP) * G::K_BYTES;
+            T *u1w = u1s + (q & 1) * (G::U1_BYTES / (int)sizeof(T));
+            T o1p[2][VEC], unp[2][VEC];
+            KW kqv[2];
+            // ---- step n+1 on plane q, rows r0, r0+1 (-1 .. TY)
+#pragma unroll
+            for (int k = 0; k < 2; k++) {
+                const int r = r0 + k, sr = r + 2;
+                T ym[VEC], yp[VEC], pv[VEC];
+                *(uint4 *)unp[k] = *(const uint4 *)(uqp + sr * UROW + col);
+                *(uint4 *)ym = *(const uint4 *)(uq + (sr - 1) * UROW + col);
+                *(uint4 *)yp = *(const uint4 *)(uq + (sr + 1) * UROW + col);
+                *(uint4 *)pv = *(const uint4 *)(pq + (r + 1) * TX + lane * VEC);
+                kqv[k] = *(const KW *)(kq + (r + 1) * G::KROW + kd + lane * VEC);
+                T left = __shfl_up_sync(0xffffffffu, unc[k][VEC - 1], 1);
+                T right = __shfl_down_sync(0xffffffffu, unc[k][0], 1);
+                if (lane == 0) left = uq[sr * UROW + VEC - 1];
+                if (lane == 31) right = uq[sr * UROW + VEC + TX];
+                vol_vec<T>(unc[k], ym, yp, unm[k], unp[k], pv, left, right, (uint32_t)kqv[k], l2, o1p[k]);
+                *(uint4 *)(u1w + (r + 1) * TX + lane * VEC) = *(const uint4 *)o1p[k];
+                if (q >= pa && q < pb && r >= 0 && r < TY && x_ok && oy + r < g.ny) {
+                    T *dst = out1 + (int64_t)q * g.plane + (int64_t)(oy + r + 1) * g.pitch + g.xo + xv;
+                    tb::st_v4_hint(dst, *(const uint4 *)o1p[k], pol);
+                }
+            }
+            __syncthreads();  // u^{n+1} of plane q complete in shared memory
+            // ---- step n+2 on plane q-1 (rows 0 .. TY-1, core lanes store)
+            if (q - 1 >= pa) {
+                const T *u1r = u1s + ((q - 1) & 1) * (G::U1_BYTES / (int)sizeof(T));
+#pragma unroll
+                for (int k = 0; k < 2; k++) {
+                    const int r = r0 + k;
+                    if (r < 0 || r >= TY) continue;  // warp-uniform
+                    T ym[VEC], yp[VEC], o2[VEC];
+                    *(uint4 *)ym = *(const uint4 *)(u1r + r * TX + lane * VEC);
+                    *(uint4 *)yp = *(const uint4 *)(u1r + (r + 2) * TX + lane * VEC);
+                    const T left = __shfl_up_sync(0xffffffffu, o1c[k][VEC - 1], 1);
+                    const T right = __shfl_down_sync(0xffffffffu, o1c[k][0], 1);
+                    vol_vec<T>(o1c[k], ym, yp, o1m[k], o1p[k], unm[k], left, right, (uint32_t)km[k], l2, o2);
+                    if (x_ok && oy + r < g.ny) {
+                        T *dst = out2 + (int64_t)(q - 1) * g.plane + (int64_t)(oy + r + 1) * g.pitch + g.xo + xv;
+                        tb::st_v4_hint(dst, *(const uint4 *)o2, pol);
+                    }
+                }
+            }
+#pragma unroll
+            for (int k = 0; k < 2; k++) {
+#pragma unroll
+                for (int i = 0; i < VEC; i++) {
+                    o1m[k][i] = o1c[k][i];
+                    o1c[k][i] = o1p[k][i];
+                    unm[k][i] = unc[k][i];
+                    unc[k][i] = unp[k][i];
+                }
+                km[k] = kqv[k];
+            }
+            __syncthreads();  // u^n(q), u^{n-1}/K(q), u^{n+1}(q-1) no longer read
+            if (tid == 0) {
+                asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+                if (q + SU <= pb + 1) issue_u(q + SU);  // into the slot of plane q
+                if (q + SP <= pb) issue_pk(q + SP);
+            }
+        }
+    }
+}
+
+// ------------------------------------------------------------------ the shell
+// shell voxel: inside, and itself or a face neighbour a boundary node
+static __device__ __forceinline__ bool is_shell(const uint8_t *K, int64_t i, const Grid &g)
+{
+    const int k = K[i];
+    if (k == 0) return false;
+    if (k < 6) return true;
+    return K[i - 1] < 6 || K[i + 1] < 6 || K[i - g.pitch] < 6 || K[i + g.pitch] < 6 || K[i - g.plane] < 6 ||
+           K[i + g.plane] < 6;
+}
+
+// per-row counts with a block reduction (one block per row)
+__global__ void k_shell_row_counts(Grid g, const uint8_t *__restrict__ K, int64_t *__restrict__ cnt)
+{
+    __shared__ int red[32];
+    const int64_t rows = (int64_t)g.lnz * g.ny;
+    for (int64_t row = blockIdx.x; row < rows; row += gridDim.x) {
+        const int64_t y = row % g.ny, z = row / g.ny;
+        const int64_t b = (z + 1) * g.plane + (y + 1) * g.pitch + g.xo;
+        int c = 0;
+        for (int x = threadIdx.x; x < g.nx; x += blockDim.x) c += is_shell(K, b + x, g);
+#pragma unroll
+        for (int o = 16; o; o >>= 1) c += __shfl_xor_sync(0xffffffffu, c, o);
+        if ((threadIdx.x & 31) == 0) red[threadIdx.x >> 5] = c;
+        __syncthreads();
+        if (threadIdx.x == 0) {
+            int s = 0;
+            for (int w = 0; w < (int)(blockDim.x >> 5); w++) s += red[w];
+            cnt[row] = s;
+        }
+        __syncthreads();
+    }
+}
+
+// ascending padded positions of the shell voxels (one block per row, a block
+// scan keeps the x order)
+template <typename IdxT>
+__global__ void k_shell_compact(Grid g, const uint8_t *__restrict__ K, const int64_t *__restrict__ off,
+                                IdxT *__restrict__ list)
+{
+    __shared__ int wsum[32];
+    __shared__ int64_t base_s;
+    const int64_t rows = (int64_t)g.lnz * g.ny;
+    const int nwarps = blockDim.x >> 5, lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+    for (int64_t row = blockIdx.x; row < rows; row += gridDim.x) {
+        const int64_t y = row % g.ny, z = row / g.ny;
+        const int64_t b = (z + 1) * g.plane + (y + 1) * g.pitch + g.xo;
+        if (threadIdx.x == 0) base_s = off[row];
+        __syncthreads();
+        for (int x0 = 0; x0 < g.nx; x0 += blockDim.x) {
+            const int x = x0 + threadIdx.x;
+            const bool f = x < g.nx && is_shell(K, b + x, g);
+            const unsigned m = __ballot_sync(0xffffffffu, f);
+            if (lane == 0) wsum[w] = __popc(m);
+            __syncthreads();
+            int before = 0, total = 0;
+            for (int k = 0; k < nwarps; k++) {
+                before += k < w ? wsum[k] : 0;
+                total += wsum[k];
+            }
+            if (f) list[base_s + before + __popc(m & ((1u << lane) - 1u))] = (IdxT)(b + x);
+            __syncthreads();
+            if (threadIdx.x == 0) base_s += total;
+            __syncthreads();
+        }
+    }
+}
+
+// u^{n+2} at the shell voxels and the source's 7-point star (src[7], -1 =
+// none), from the final u^{n+1} (u1) and u^n (u0): the volume update in the
+// order of DESIGN.md §4 (same expression as vol_vec).
+template <typename T, typename IdxT>
+__global__ void __launch_bounds__(256) k_shell(const IdxT *__restrict__ list, int64_t n, const int64_t *__restrict__ src,
+                                               const T *__restrict__ u1, const T *__restrict__ u0,
+                                               const uint8_t *__restrict__ K, T *__restrict__ out, Grid g, T l2)
+{
+    using R = rn<T>;
+    const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (i >= n + 7) return;
+    const int64_t p = i < n ? (int64_t)list[i] : src[i - n];
+    if (p < 0) return;
+    const int nbr = K[p];
+    if (nbr == 0) return;
+    T s = R::add(u1[p - 1], u1[p + 1]);
+    s = R::add(s, u1[p - g.pitch]);
+    s = R::add(s, u1[p + g.pitch]);
+    s = R::add(s, u1[p - g.plane]);
+    s = R::add(s, u1[p + g.plane]);
+    const T a = R::sub((T)2, R::mul(l2, (T)nbr));
+    T t = R::mul(a, u1[p]);
+    t = R::add(t, R::mul(l2, s));
+    out[p] = R::sub(t, u0[p]);
+}
+
+// ------------------------------------------------------------------ host side
+static PFN_cuTensorMapEncodeTiled_v12000 tb_encode_fn()
+{
+    static PFN_cuTensorMapEncodeTiled_v12000 fn = nullptr;
+    if (!fn) {
+        cudaDriverEntryPointQueryResult q;
+        void *p = nullptr;
+        if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &p, cudaEnableDefault, &q) == cudaSuccess &&
+            q == cudaDriverEntryPointSuccess)
+            fn = (PFN_cuTensorMapEncodeTiled_v12000)p;
+    }
+    return fn;
+}
+
+static bool tb_map(CUtensorMap *m, CUtensorMapDataType dt, size_t esize, void *base, const Grid &g, int bx, int by,
+                   int xpad = 0)
+{
+    auto fn = tb_encode_fn();
+    if (!fn) return false;
+    cuuint64_t dims[3] = {(cuuint64_t)(g.pitch + xpad), (cuuint64_t)(g.ny + 2), (cuuint64_t)(g.lnz + 2)};
+    cuuint64_t strides[2] = {(cuuint64_t)(g.pitch * esize), (cuuint64_t)(g.plane * esize)};
+    cuuint32_t box[3] = {(cuuint32_t)bx, (cuuint32_t)by, 1};
+    cuuint32_t es[3] = {1, 1, 1};
+    return fn(m, dt, 3, base, dims, strides, box, es, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE,
+              CU_TENSOR_MAP_L2_PROMOTION_L2_128B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
+}
+
+static constexpr int kTbTY = 32, kTbSU = 4, kTbSP = 3;
+
+struct TwoStepPlan {
+    CUtensorMap umap[4], pmap[4], kmap;
+    int tiles_x, tiles_y, grid, smem;
+    void *list = nullptr;  // shell positions (uint32 or int64), ascending
+    int64_t n_shell = 0;
+    int64_t *src = nullptr;  // [7] the source's star, -1 = none
+    bool idx64 = false;
+};
+
+template <typename T>
+cudaError_t twostep_plan_create(const Grid &g, void *const u[4], uint8_t *K_alloc, const uint8_t *K, bool idx64,
+                                int nsm, cudaStream_t s, void **plan_out, int64_t *n_shell)
+{
+    using G = TbGeom<T, kTbTY, kTbSU, kTbSP>;
+    auto *pl = new TwoStepPlan();
+    const CUtensorMapDataType dt = sizeof(T) == 4 ? CU_TENSOR_MAP_DATA_TYPE_FLOAT32 : CU_TENSOR_MAP_DATA_TYPE_FLOAT64;
+    bool ok = true;
+    for (int k = 0; k < 4; k++) {
+        ok = ok && tb_map(&pl->umap[k], dt, sizeof(T), u[k], g, G::UROW, G::UR);
+        ok = ok && tb_map(&pl->pmap[k], dt, sizeof(T), u[k], g, G::TX, G::PR);
+    }
+    ok = ok && tb_map(&pl->kmap, CU_TENSOR_MAP_DATA_TYPE_UINT8, 1, K_alloc, g, G::KROW, G::PR, k_shift(g));
+    if (!ok) {
+        delete pl;
+        return cudaErrorNotSupported;
+    }
+    pl->tiles_x = (g.nx + G::TXO - 1) / G::TXO;
+    pl->tiles_y = (g.ny + kTbTY - 1) / kTbTY;
+    pl->smem = G::SMEM;
+    pl->idx64 = idx64;
+    auto kern = k_volume2<T, kTbTY, kTbSU, kTbSP>;
+    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, pl->smem);
+    int occ = 0;
+    if (e == cudaSuccess) e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kern, G::NT, pl->smem);
+    if (e == cudaSuccess && occ < 1) e = cudaErrorInvalidConfiguration;
+    pl->grid = nsm * std::max(occ, 1);
+    // the shell list
+    const int64_t rows = (int64_t)g.lnz * g.ny;
+    int64_t *cnt = nullptr, *off = nullptr;
+    void *tmp = nullptr;
+    size_t tb = 0;
+    if (e == cudaSuccess) e = cudaMalloc(&cnt, (size_t)(rows + 1) * 8);
+    if (e == cudaSuccess) e = cudaMalloc(&off, (size_t)(rows + 1) * 8);
+    if (e == cudaSuccess) e = cudaMemsetAsync(cnt, 0, (size_t)(rows + 1) * 8, s);
+    const unsigned blocks = (unsigned)std::max<int64_t>(1, std::min<int64_t>(rows, (int64_t)nsm * 16));
+    if (e == cudaSuccess && rows > 0) {
+        k_shell_row_counts<<<blocks, 256, 0, s>>>(g, K, cnt);
+        e = cudaGetLastError();
+    }
+    if (e == cudaSuccess) e = exclusive_scan_rows64(cnt, off, rows + 1, nullptr, &tb, s);
+    if (e == cudaSuccess) e = cudaMalloc(&tmp, tb ? tb : 16);
+    if (e == cudaSuccess) e = exclusive_scan_rows64(cnt, off, rows + 1, tmp, &tb, s);
+    int64_t n = 0;
+    if (e == cudaSuccess) e = cudaMemcpyAsync(&n, off + rows, 8, cudaMemcpyDeviceToHost, s);
+    if (e == cudaSuccess) e = cudaStreamSynchronize(s);
+    if (e == cudaSuccess) e = cudaMalloc(&pl->list, (size_t)std::max<int64_t>(n, 1) * (idx64 ? 8 : 4));
+    if (e == cudaSuccess && rows > 0 && n > 0) {
+        if (idx64) k_shell_compact<int64_t><<<blocks, 256, 0, s>>>(g, K, off, (int64_t *)pl->list);
+        else k_shell_compact<uint32_t><<<blocks, 256, 0, s>>>(g, K, off, (uint32_t *)pl->list);
+        e = cudaGetLastError();
+    }
+    if (e == cudaSuccess) e = cudaMalloc(&pl->src, 7 * 8);
+    if (e == cudaSuccess) e = cudaMemsetAsync(pl->src, 0xff, 7 * 8, s);
+    if (e == cudaSuccess) e = cudaStreamSynchronize(s);
+    if (cnt) cudaFree(cnt);
+    if (off) cudaFree(off);
+    if (tmp) cudaFree(tmp);
+    pl->n_shell = n;
+    if (e != cudaSuccess) {
+        if (pl->list) cudaFree(pl->list);
+        if (pl->src) cudaFree(pl->src);
+        delete pl;
+        return e;
+    }
+    *n_shell = n;
+    *plan_out = pl;
+    return cudaSuccess;
+}
+
+void twostep_plan_destroy(void *plan)
+{
+    auto *pl = (TwoStepPlan *)plan;
+    if (!pl) return;
+    if (pl->list) cudaFree(pl->list);
+    if (pl->src) cudaFree(pl->src);
+    delete pl;
+}
+
+cudaError_t twostep_set_source(void *plan, int64_t pos, const Grid &g)
+{
+    auto *pl = (TwoStepPlan *)plan;
+    int64_t h[7];
+    for (int k = 0; k < 7; k++) h[k] = -1;
+    if (pos >= 0) {
+        const int64_t d[7] = {0, -1, 1, -g.pitch, g.pitch, -g.plane, g.plane};
+        for (int k = 0; k < 7; k++) h[k] = pos + d[k];
+    }
+    return cudaMemcpy(pl->src, h, sizeof h, cudaMemcpyHostToDevice);
+}
+
+static int tb_choose_zchunk(int nz, int tiles, int grid)
+{
+    long best = -1;
+    int best_c = nz;
+    for (int n = 1; n <= nz; n++) {
+        const int c = (nz + n - 1) / n;
+        const long units = (long)tiles * ((nz + c - 1) / c);
+        const long rounds = (units + grid - 1) / grid;
+        const long cost = rounds * (c + 4);  // +4: the z ring recomputed / re-read per chunk
+        if (best < 0 || cost < best) {
+            best = cost;
+            best_c = c;
+        }
+        if (c == 1) break;
+    }
+    return best_c;
+}
+
+template <typename T>
+cudaError_t launch_volume2(const void *plan, const Grid &g, int cur_buf, int prev_buf, T *out1, T *out2,
+                           double lambda, cudaStream_t s)
+{
+    using G = TbGeom<T, kTbTY, kTbSU, kTbSP>;
+    const auto *pl = (const TwoStepPlan *)plan;
+    if (g.lnz <= 0) return cudaSuccess;
+    const T l2 = (T)(lambda * lambda);
+    const int tiles = pl->tiles_x * pl->tiles_y;
+    const int zc = tb_choose_zchunk(g.lnz, tiles, pl->grid);
+    const long units = (long)tiles * ((g.lnz + zc - 1) / zc);
+    const int grid = (int)std::min<long>(pl->grid, units);
+    k_volume2<T, kTbTY, kTbSU, kTbSP><<<grid, G::NT, pl->smem, s>>>(pl->umap[cur_buf], pl->pmap[prev_buf], pl->kmap,
+                                                                    out1, out2, g, l2, zc, pl->tiles_x, pl->tiles_y);
+    return cudaGetLastError();
+}
+
+template <typename T>
+cudaError_t launch_shell(const void *plan, const Grid &g, const T *u1, const T *u0, const uint8_t *K, T *out,
+                         double lambda, cudaStream_t s)
+{
+    const auto *pl = (const TwoStepPlan *)plan;
+    const T l2 = (T)(lambda * lambda);
+    const int64_t n = pl->n_shell + 7;
+    const unsigned blocks = (unsigned)((n + 255) / 256);
+    if (pl->idx64)
+        k_shell<T, int64_t><<<blocks, 256, 0, s>>>((const int64_t *)pl->list, pl->n_shell, pl->src, u1, u0, K, out,
+                                                   g, l2);
+    else
+        k_shell<T, uint32_t><<<blocks, 256, 0, s>>>((const uint32_t *)pl->list, pl->n_shell, pl->src, u1, u0, K, out,
+                                                    g, l2);
+    return cudaGetLastError();
+}
+
+#define RAFD_TB_INST(T)                                                                                            \
+    template cudaError_t twostep_plan_create<T>(const Grid &, void *const[4], uint8_t *, const uint8_t *, bool, int, \
+                                                cudaStream_t, void **, int64_t *);                                  \
+    template cudaError_t launch_volume2<T>(const void *, const Grid &, int, int, T *, T *, double, cudaStream_t);   \
+    template cudaError_t launch_shell<T>(const void *, const Grid &, const T *, const T *, const uint8_t *, T *,     \
+                                         double, cudaStream_t);
+RAFD_TB_INST(float)
+RAFD_TB_INST(double)
+#undef RAFD_TB_INST
+
+}  // namespace rafd

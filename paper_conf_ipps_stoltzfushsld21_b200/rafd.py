@@ -37,7 +37,7 @@ ABI_SYMBOLS = [
     "rafd_read_branch_state", "rafd_get_classification", "rafd_get_info", "rafd_energy",
     "rafd_set_profiling", "rafd_get_kernel_times", "rafd_launch_count", "rafd_slab_plan",
     "rafd_nccl_unique_id", "rafd_last_error", "rafd_strerror", "rafd_version",
-    "rafd_ipc_handle", "rafd_ipc_connect", "rafd_set_step",
+    "rafd_ipc_handle", "rafd_ipc_connect", "rafd_set_step", "rafd_set_temporal_blocking",
 ]
 RAFD_IPC_BLOB_BYTES = 208
 
@@ -65,13 +65,15 @@ class rafd_info(C.Structure):
                 ("boundary_bytes", C.c_int64), ("device_bytes", C.c_int64),
                 ("precision", C.c_int32), ("n_materials", C.c_int32), ("n_branches", C.c_int32),
                 ("z_begin", C.c_int32), ("z_end", C.c_int32), ("pitch", C.c_int32),
-                ("fused", C.c_int32), ("scheme", C.c_int32)]
+                ("fused", C.c_int32), ("scheme", C.c_int32), ("steps_per_sweep", C.c_int32),
+                ("reserved_", C.c_int32), ("n_shell", C.c_int64)]
 
 
 class rafd_kernel_times(C.Structure):
     _fields_ = [("volume_ms", C.c_double), ("boundary_ms", C.c_double), ("other_ms", C.c_double),
                 ("volume_launches", C.c_int64), ("boundary_launches", C.c_int64),
-                ("other_launches", C.c_int64)]
+                ("other_launches", C.c_int64), ("shell_ms", C.c_double),
+                ("shell_launches", C.c_int64)]
 
 
 _lib = None
@@ -95,6 +97,7 @@ def lib():
     L.rafd_set_receivers.argtypes = [P, I32, P]
     L.rafd_set_state.argtypes = [P, P, P, P, P]
     L.rafd_step.argtypes = [P, I64]
+    L.rafd_set_temporal_blocking.argtypes = [P, I32]
     L.rafd_set_step.argtypes = [P, I64]
     L.rafd_step_group.argtypes = [C.POINTER(P), I32, I64]
     L.rafd_synchronize.argtypes = [P]
@@ -234,6 +237,10 @@ class Room:
     # --- run
     def step(self, n):
         _check(lib().rafd_step(self.h, int(n)))
+
+    def set_temporal_blocking(self, steps_per_sweep):
+        """rafd_set_temporal_blocking: 2 = two leapfrog steps per grid sweep."""
+        _check(lib().rafd_set_temporal_blocking(self.h, int(steps_per_sweep)))
 
     def synchronize(self):
         _check(lib().rafd_synchronize(self.h))
