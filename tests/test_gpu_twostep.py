@@ -57,7 +57,9 @@ def compare(o, g, precision, branches=False):
     cg, pg = g.read_field()
     assert_same(co, cg, precision, "u^n")
     assert_same(po, pg, precision, "u^{n-1}")
-    assert_same(o.read_receivers(), g.read_receivers(), precision, "receivers")
+    ro, rg = o.read_receivers(), g.read_receivers()
+    if ro.size or rg.size:
+        assert_same(ro, rg, precision, "receivers")
     if branches:
         vo, go = o.read_branch_state()
         vg, gg = g.read_branch_state()
