@@ -277,11 +277,13 @@ def run_rafd(args, rank, world, local_rank):
         bnd_gbs = info["boundary_bytes"] / (bnd_ms * 1e-3) / 1e9 if (info["n_boundary"] and bnd_ms > 0) else None
         step_gbs = bytes_total * args.steps / (ms_max * 1e-3) / 1e9 / world
         traffic = None
-        tp = os.path.join(ROOT, "profiles", "volume_traffic.json")
+        # ncu DRAM bytes of one launch of the timed kernel on this config (committed under profiles/)
+        tp = os.path.join(ROOT, "profiles", "volume2_traffic.json" if tb == 2 else "volume_traffic.json")
         if os.path.exists(tp):
             try:
                 tj = json.load(open(tp))
-                if bool(tj.get("fused", False)) == fused and args.config == "C4" and world == 1:
+                if bool(tj.get("fused", False)) == fused and args.config == "C4" and world == 1 \
+                        and tj.get("precision", 32) == prec:
                     traffic = tj.get("dram_bytes_per_launch")
             except Exception:
                 traffic = None

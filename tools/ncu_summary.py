@@ -36,11 +36,11 @@ def launches(path):
             continue
         if hdr and len(r) == len(hdr):
             d = dict(zip(hdr, r))
-            name = re.sub(r"\(.*", "", d["Kernel Name"]).replace("void ", "")
+            name = re.sub(r"\(.*", "", d["Kernel Name"]).replace("void ", "").replace("rafd::", "")
             ns = float(d["Metric Value"]) * (1e3 if d["Metric Unit"] == "usecond" else 1e6 if d["Metric Unit"] == "msecond" else 1)
             per[name].append(ns)
             order.append(name)
-    step = [k for k in per if k.startswith("rafd::k_volume") or k.startswith("rafd::k_boundary") or k.startswith("rafd::k_src")]
+    step = [k for k in per if k.startswith(("k_volume", "k_boundary", "k_src", "k_shell<"))]
     tot = sum(sum(per[k]) for k in step)
     out = {"kernels": {}, "note": "ncu --metrics gpu__time_duration.sum --clock-control none: cold-cache, serialised; compare shares"}
     for k in step:
