@@ -2,8 +2,10 @@
 the C4 hall (1536x1024x704 = 1.107e9 voxels, FD-MM MB=3, M=8, fp32), default
 volume-kernel tiling, inputs generated on the device exactly as bench.py does.
 From a seeded random state (fields and branch state) both the CUDA path and
-the oracle take 2 steps; every voxel, every branch state and the receivers are
-compared bit for bit.  Host memory ~40 GB, ~1-2 min."""
+the oracle take 2 steps -- the CUDA path once with single steps and once with
+temporal blocking (one double step of k_volume2 + shell, the bench default) --
+and every voxel, every branch state and the receivers are compared bit for
+bit.  Host memory ~40 GB, ~1-2 min."""
 import math
 
 import numpy as np
@@ -25,18 +27,21 @@ def test_c4_full_size_two_steps_bitwise(orc):
     dev = torch.device("cuda", 0)
     mask_d, mm_d, _ = bench.slab_inputs(cfg, 0, nz, dev)
     g = rafd.Room(mask_d, LAM, 32, beta0, D, E, F, matmap=mm_d)
+    g2 = rafd.Room(mask_d, LAM, 32, beta0, D, E, F, matmap=mm_d)
+    g2.set_temporal_blocking(2)
     nb = g.nb
     gen = torch.Generator(device=dev).manual_seed(20251017)
     up = torch.rand((nz, ny, nx), generator=gen, device=dev, dtype=torch.float32) * 2 - 1
     uc = torch.rand((nz, ny, nx), generator=gen, device=dev, dtype=torch.float32) * 2 - 1
     v0 = (torch.rand((3, nb), generator=gen, device=dev, dtype=torch.float32) - 0.5) * 0.2
     g0 = (torch.rand((3, nb), generator=gen, device=dev, dtype=torch.float32) - 0.5) * 0.2
-    g.set_state(up, uc, v0, g0)
     src = I.source_position((nx, ny, nz))
     rcv = I.receiver_positions((nx, ny, nz))
-    g.set_source(src, [1.0, -0.5])
-    g.set_receivers(rcv)
-    g.step(2)
+    for r in (g, g2):
+        r.set_state(up, uc, v0, g0)
+        r.set_source(src, [1.0, -0.5])
+        r.set_receivers(rcv)
+        r.step(2)
 
     o = orc.OracleRoom(mask_d.cpu().numpy(), LAM, 32, beta0, D, E, F, matmap=mm_d.cpu().numpy())
     del mask_d, mm_d
@@ -47,16 +52,19 @@ def test_c4_full_size_two_steps_bitwise(orc):
     o.set_receivers(rcv)
     o.step(2)
 
-    cur_g = torch.empty((nz, ny, nx), dtype=torch.float32, device=dev)
-    prv_g = torch.empty_like(cur_g)
-    g.read_field(out_curr=cur_g, out_prev=prv_g)
     cur_o, prv_o = o.read_field()
-    assert np.array_equal(cur_g.cpu().numpy(), cur_o)
-    assert np.array_equal(prv_g.cpu().numpy(), prv_o)
-    vg, gg = g.read_branch_state()
     vo, go = o.read_branch_state()
-    assert np.array_equal(vg, vo) and np.array_equal(gg, go)
-    assert np.array_equal(g.read_receivers(), o.read_receivers())
+    rec_o = o.read_receivers()
+    for r in (g, g2):
+        cur_g = torch.empty((nz, ny, nx), dtype=torch.float32, device=dev)
+        prv_g = torch.empty_like(cur_g)
+        r.read_field(out_curr=cur_g, out_prev=prv_g)
+        assert np.array_equal(cur_g.cpu().numpy(), cur_o)
+        assert np.array_equal(prv_g.cpu().numpy(), prv_o)
+        del cur_g, prv_g
+        vg, gg = r.read_branch_state()
+        assert np.array_equal(vg, vo) and np.array_equal(gg, go)
+        assert np.array_equal(r.read_receivers(), rec_o)
 
 
 @pytest.mark.parametrize("name,precision,steps", [("C2a", 32, 30), ("C2b", 32, 30), ("C3", 32, 12), ("C3d", 64, 12)])
@@ -64,7 +72,7 @@ def test_config_full_size_bitwise(orc, name, precision, steps):
     """BASELINE.json configs[1..2] at full size (256^3 L-shape and dome with
     FI-MM M=4; 512x384x256 box with FD-MM MB=3 M=8 in fp32 and fp64): a few
     steps from a seeded random state plus the config's source, every voxel and
-    the receivers bitwise."""
+    the receivers bitwise -- with single steps and with temporal blocking."""
     cfg = I.CONFIGS[name]
     nx, ny, nz = cfg["dims"]
     mask_t = I.make_mask(cfg["shape"], nx, ny, nz)
@@ -72,6 +80,8 @@ def test_config_full_size_bitwise(orc, name, precision, steps):
     mask = mask_t.numpy()
     beta0, D, E, F = I.config_materials(cfg)
     g = rafd.Room(mask, LAM, precision, beta0, D, E, F, matmap=mm)
+    g2 = rafd.Room(mask, LAM, precision, beta0, D, E, F, matmap=mm)
+    g2.set_temporal_blocking(2)
     o = orc.OracleRoom(mask, LAM, precision, beta0, D, E, F, matmap=mm)
     dt = np.float32 if precision == 32 else np.float64
     rng = np.random.default_rng(7)
@@ -79,17 +89,22 @@ def test_config_full_size_bitwise(orc, name, precision, steps):
     uc = rng.uniform(-1, 1, mask.shape).astype(dt)
     src = I.source_position(cfg["dims"], mask)
     rcv = I.receiver_positions(cfg["dims"], mask)
-    for r in (g, o):
+    for r in (g, g2, o):
         r.set_state(up, uc)
         r.set_source(src, I.impulse())
         r.set_receivers(rcv)
-        r.step(steps)
-    assert np.array_equal(g.read_field()[0], o.read_field()[0])
-    assert np.array_equal(g.read_receivers(), o.read_receivers())
+        r.step(steps + 1)  # odd: the two-step room ends with one single step
+    fo = o.read_field()[0]
+    assert np.array_equal(g.read_field()[0], fo)
+    assert np.array_equal(g2.read_field()[0], fo)
+    ro = o.read_receivers()
+    assert np.array_equal(g.read_receivers(), ro)
+    assert np.array_equal(g2.read_receivers(), ro)
     if cfg["MB"]:
-        vg, gg = g.read_branch_state()
         vo, go = o.read_branch_state()
-        assert np.array_equal(vg, vo) and np.array_equal(gg, go)
+        for r in (g, g2):
+            vg, gg = r.read_branch_state()
+            assert np.array_equal(vg, vo) and np.array_equal(gg, go)
 
 
 def test_c5_hall_int64_indexing_light_cone():
