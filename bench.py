@@ -170,11 +170,15 @@ def bench_device(local_rank):
     return int(d) if d is not None else local_rank
 
 
-def connect_ipc(room, rank, world):
-    """Exchange the slabs' CUDA-IPC blobs and connect neighbours (transport 'ipc')."""
+def connect_ipc(room, rank, world, push=False):
+    """Exchange the slabs' CUDA-IPC blobs and connect neighbours (transports
+    'ipc': copy pulls; 'push': the edge-phase kernels store into the
+    neighbours' ghost planes)."""
     blobs = [None] * world
     torch.distributed.all_gather_object(blobs, room.ipc_handle())
     room.ipc_connect(blobs[rank - 1] if rank > 0 else None, blobs[rank + 1] if rank < world - 1 else None)
+    if push:
+        room.set_halo_push(True)
     torch.distributed.barrier()
 
 
@@ -204,8 +208,8 @@ def run_rafd(args, rank, world, local_rank):
     room = rafd.Room(mask, LAM, prec, beta0, D, E, F, matmap=mm, device=local_rank,
                      stream=stream.cuda_stream, rank=rank, nranks=world, nccl_id=nccl_id,
                      z_begin=z0, z_end=z1, mask_z0=mz0, dims=(nx, ny, nz))
-    if world > 1 and args.transport == "ipc":
-        connect_ipc(room, rank, world)
+    if world > 1 and args.transport in ("ipc", "push"):
+        connect_ipc(room, rank, world, push=args.transport == "push")
     tb = args.tb if world == 1 else 1  # temporal blocking: whole rooms on one GPU
     if tb == 2:
         room.set_temporal_blocking(2)
@@ -363,7 +367,7 @@ def run_e2e(args, cfg, prec, beta0, D, E, F, rank, world, local_rank, plan, mult
         obj = [rafd.rafd_nccl_unique_id() if rank == 0 else None]
         torch.distributed.broadcast_object_list(obj, src=0)
         nccl_id = obj[0]
-    ipc = world > 1 and args.transport == "ipc"
+    ipc = world > 1 and args.transport in ("ipc", "push")
     sig = I.impulse()
     mask_np = None if cfg["shape"] == "box" else I.make_mask(cfg["shape"], nx, ny, nz).numpy()
     rcv = I.receiver_positions((nx, ny, nz), mask_np)
@@ -376,7 +380,7 @@ def run_e2e(args, cfg, prec, beta0, D, E, F, rank, world, local_rank, plan, mult
                      rank=rank, nranks=world, nccl_id=nccl_id, z_begin=z0, z_end=z1, mask_z0=mz0,
                      dims=(nx, ny, nz))
     if ipc:
-        connect_ipc(room, rank, world)
+        connect_ipc(room, rank, world, push=args.transport == "push")
     room.set_source(I.source_position((nx, ny, nz), mask_np), sig)
     room.set_receivers(rcv)
     tb = args.tb if world == 1 else 1
@@ -479,7 +483,7 @@ def main():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--tb", type=int, default=2, choices=[1, 2],
                     help="steps per HBM sweep (temporal blocking; whole rooms on one GPU only)")
-    ap.add_argument("--transport", default="nccl", choices=["nccl", "ipc"],
+    ap.add_argument("--transport", default="nccl", choices=["nccl", "ipc", "push"],
                     help="halo exchange for --gpus > 1: NCCL send/recv, or CUDA-IPC peer copies "
                          "ordered by GPU-side stream waits (rafd_ipc_connect)")
     args = ap.parse_args()

@@ -212,6 +212,22 @@ int rafd_step_group(rafd_room **rooms, int32_t n, int64_t nsteps);
 int rafd_ipc_handle(rafd_room *r, uint8_t *blob);
 int rafd_ipc_connect(rafd_room *r, const uint8_t *lower, const uint8_t *upper);
 
+/* Device-initiated halo for IPC-connected slabs: instead of
+ * pulling the neighbours' edge planes with copies, the kernels that produce a
+ * slab's first and last owned planes -- the volume kernel (Listing 2,
+ * PAPER.md:349-357) over those planes, the boundary kernel (Listings 3/4,
+ * PAPER.md:371-377, 415-440) over their nodes, the source -- also store every
+ * value into the neighbour's ghost plane through the peer-mapped buffer, then
+ * one GPU-side signal (a stream write with a memory fence) publishes the step.
+ * The next step waits for the neighbours' signal of the previous step, which
+ * orders both the ghost reads (RAW) and the next pushes (WAR).  Results are
+ * bitwise those of the pull transport and of the undivided room.  on = 0
+ * selects the pull transport.  Call after rafd_ipc_connect, before the first
+ * step; every slab of the room must choose the same transport.  Errors: STATE
+ * (not IPC-connected, a fused or single-kernel scheme, the v0 kernel, steps
+ * already taken), INVAL. */
+int rafd_set_halo_push(rafd_room *r, int32_t on);
+
 /* Wait for all enqueued work of the room. */
 int rafd_synchronize(rafd_room *r);
 

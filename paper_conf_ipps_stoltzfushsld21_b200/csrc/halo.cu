@@ -294,6 +294,21 @@ cudaError_t ipc_wait_peers(HaloIpc *h, int word, int64_t value, cudaStream_t s)
     return cudaSuccess;
 }
 
+// halo push (device-initiated): byte offsets that take an address in my
+// buffer `buf` to the same voxel in a neighbour's ghost plane of its buffer
+// `buf` -- my first owned plane (padded 1) -> the lower neighbour's top ghost
+// (its padded lnz_lo + 1); my last (padded lnz) -> the upper neighbour's
+// bottom ghost (padded 0).  0 where there is no neighbour.
+void ipc_mirror_deltas(HaloIpc *h, int buf, const void *mine, size_t plane_bytes, int lnz, int64_t *d_lo,
+                       int64_t *d_hi)
+{
+    *d_lo = *d_hi = 0;
+    if (h->lo.open)
+        *d_lo = (int64_t)((uintptr_t)h->lo.u[buf] - (uintptr_t)mine) + (int64_t)h->lo.lnz * (int64_t)plane_bytes;
+    if (h->hi.open)
+        *d_hi = (int64_t)((uintptr_t)h->hi.u[buf] - (uintptr_t)mine) - (int64_t)lnz * (int64_t)plane_bytes;
+}
+
 // ghost planes of my buffer `buf` <- the neighbours' edge planes of their buffer `buf`
 // (all slabs step in lock-step, so they use the same buffer parity)
 cudaError_t ipc_pull(HaloIpc *h, int buf, void *mine, size_t plane_bytes, int lnz, cudaStream_t s)

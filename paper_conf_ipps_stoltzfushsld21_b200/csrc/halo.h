@@ -37,4 +37,6 @@ void ipc_close(HaloIpc *h);
 cudaError_t ipc_signal(int64_t *addr, int64_t value, cudaStream_t s);
 cudaError_t ipc_wait_peers(HaloIpc *h, int word, int64_t value, cudaStream_t s);
 cudaError_t ipc_pull(HaloIpc *h, int buf, void *mine, size_t plane_bytes, int lnz, cudaStream_t s);
+void ipc_mirror_deltas(HaloIpc *h, int buf, const void *mine, size_t plane_bytes, int lnz, int64_t *d_lo,
+                       int64_t *d_hi);
 }  // namespace rafd

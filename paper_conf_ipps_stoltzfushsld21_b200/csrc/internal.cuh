@@ -81,6 +81,9 @@ template <typename T> struct FusedArgs {
     T beta1;         // Listing 1 admittance
     T loss1, loss2;  // Listing 6 constants
     const uint8_t *occ;  // [lnz+2][tiles] tile-plane occupancy (set by the plan), or nullptr
+    // halo push: byte offsets from an output address to the
+    // same voxel in a neighbour's ghost plane (peer memory); 0 = no mirror
+    int64_t mirror[2];
 };
 
 // plan == nullptr selects the one-thread-per-voxel v0 kernel (A/B reference);
@@ -114,9 +117,11 @@ cudaError_t launch_shell(const void *plan, const Grid &g, const T *u1, const T *
 template <typename T>
 cudaError_t launch_boundary(int MB, bool idx64, const void *bpos, const uint8_t *Kb,
                             const uint8_t *matb, int64_t i_lo, int64_t i_hi, int64_t Nb, T *unext,
-                            T *ub, T *g, T *v, const T *tab, int M, double lambda, cudaStream_t s);
+                            T *ub, T *g, T *v, const T *tab, int M, double lambda, cudaStream_t s,
+                            int64_t mirror0 = 0, int64_t mirror1 = 0);
 template <typename T>
-cudaError_t launch_src_rcv(T *unext, T *ub, Ctl<T> *ctl, cudaStream_t s, int mode = 3);
+cudaError_t launch_src_rcv(T *unext, T *ub, Ctl<T> *ctl, cudaStream_t s, int mode = 3, int64_t mirror0 = 0,
+                           int64_t mirror1 = 0);
 cudaError_t launch_find_node(const void *bpos, bool idx64, int64_t Nb, int64_t pos, int64_t *out,
                              cudaStream_t s);
 

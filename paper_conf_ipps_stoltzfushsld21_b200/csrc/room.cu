@@ -141,6 +141,7 @@ struct rafd_room {
     Halo *halo = nullptr;
     bool local_slab = false;
     HaloIpc *ipc = nullptr;   // cross-process slabs (rafd_ipc_connect)
+    bool push = false;        // IPC halo pushed by the edge-phase kernels (rafd_set_halo_push)
     int64_t *ipc_sig = nullptr;  // [2] IPC signal words (edge done, pulls done)
     // edge-first step of a slab: edge planes, then the halo exchange on
     // comm_stream overlapped with the interior planes
@@ -772,7 +773,10 @@ template <typename T> static cudaError_t enqueue_step2(rafd_room *r, int pair, i
 // last owned plane (volume, their boundary nodes, the source if it lies there),
 // then the halo exchange runs on comm_stream while phase 1 = the interior
 // planes (volume, boundary nodes, source, receivers) runs on the main stream.
-template <typename T> static cudaError_t enqueue_phase(rafd_room *r, int phase, cudaStream_t s, bool prof)
+// mirror (halo push): byte offsets to the lower / upper neighbour's ghost plane
+// for the phase-0 stores (null = no push)
+template <typename T>
+static cudaError_t enqueue_phase(rafd_room *r, int phase, cudaStream_t s, bool prof, const int64_t *mirror = nullptr)
 {
     const Grid &g = r->g;
     const int lnz = g.lnz, cur = r->cur;
@@ -790,32 +794,40 @@ template <typename T> static cudaError_t enqueue_phase(rafd_room *r, int phase, 
         return e;
     };
     const FusedArgs<T> fa = fused_args<T>(r);
-    auto vol = [&](int zl, int zh) {
+    // mirrors of the first owned plane (to the lower neighbour) and the last (to the upper one)
+    const int64_t m_lo = mirror ? mirror[0] : 0, m_hi = mirror ? mirror[1] : 0;
+    const int64_t mf0 = m_lo, mf1 = lnz == 1 ? m_hi : 0;  // plane 0 (and the last, if it is the same)
+    auto vol = [&](int zl, int zh, int64_t m0, int64_t m1) {
+        FusedArgs<T> f = fa;
+        f.mirror[0] = m0;
+        f.mirror[1] = m1;
         return timed(0, [&] {
             return launch_volume<T>(g, uc, un, r->K, r->lambda, zl, zh, s, r->vplan, cur,
-                                    (r->fused || r->scheme) ? &fa : nullptr);
+                                    (r->fused || r->scheme || m0 || m1) ? &f : nullptr);
         });
     };
-    auto bnd = [&](int64_t lo, int64_t hi) -> cudaError_t {
+    auto bnd = [&](int64_t lo, int64_t hi, int64_t m0, int64_t m1) -> cudaError_t {
         if (hi <= lo || r->fused || r->scheme) return cudaSuccess;
         return timed(1, [&] {
             return launch_boundary<T>(r->MB, r->idx64, r->bpos, r->Kb, r->matb, lo, hi, r->nb, un,
                                       ub_slot<T>(r, cur), (T *)r->gst, (T *)r->vst, (const T *)r->tab, r->M,
-                                      r->lambda, s);
+                                      r->lambda, s, m0, m1);
         });
     };
     const int zs = r->src_z >= 0 ? r->src_z - r->z0 : -1;
     const bool src_edge = zs == 0 || zs == lnz - 1;
     cudaError_t e = cudaSuccess;
     if (phase == 0) {
-        e = vol(0, 1);
-        if (e == cudaSuccess && lnz > 1) e = vol(lnz - 1, lnz);
-        if (e == cudaSuccess) e = bnd(0, std::min(r->n_first_plane, r->nb));
-        if (e == cudaSuccess && lnz > 1) e = bnd(std::max(r->n_last_start, r->n_first_plane), r->nb);
-        if (e == cudaSuccess && src_edge) e = timed(2, [&] { return launch_src_rcv<T>(un, ub_slot<T>(r, cur), ctl_of<T>(r), s, 1); });
+        e = vol(0, 1, mf0, mf1);
+        if (e == cudaSuccess && lnz > 1) e = vol(lnz - 1, lnz, m_hi, 0);
+        if (e == cudaSuccess) e = bnd(0, std::min(r->n_first_plane, r->nb), mf0, mf1);
+        if (e == cudaSuccess && lnz > 1) e = bnd(std::max(r->n_last_start, r->n_first_plane), r->nb, m_hi, 0);
+        const int64_t ms0 = zs == 0 ? mf0 : m_hi, ms1 = zs == 0 ? mf1 : 0;
+        if (e == cudaSuccess && src_edge)
+            e = timed(2, [&] { return launch_src_rcv<T>(un, ub_slot<T>(r, cur), ctl_of<T>(r), s, 1, ms0, ms1); });
     } else {
-        if (lnz > 2) e = vol(1, lnz - 1);
-        if (e == cudaSuccess && lnz > 2) e = bnd(r->n_first_plane, r->n_last_start);
+        if (lnz > 2) e = vol(1, lnz - 1, 0, 0);
+        if (e == cudaSuccess && lnz > 2) e = bnd(r->n_first_plane, r->n_last_start, 0, 0);
         if (e == cudaSuccess) e = timed(2, [&] { return launch_src_rcv<T>(un, ub_slot<T>(r, cur), ctl_of<T>(r), s, src_edge ? 2 : 3); });
     }
     return e;
@@ -851,6 +863,25 @@ template <typename T> static cudaError_t enqueue_step_ipc(rafd_room *r, bool pro
     if ((e = cudaEventRecord(r->ev_halo, r->comm_stream)) != cudaSuccess) return e;
     if ((e = enqueue_phase<T>(r, 1, r->stream, prof)) != cudaSuccess) return e;
     return cudaStreamWaitEvent(r->stream, r->ev_halo, 0);
+}
+
+// one IPC step with the halo pushed by the edge-phase kernels themselves
+// (SURVEY §8(f) f2): their stores of the first / last owned plane also go to
+// the neighbours' ghost planes over peer memory, then one signal.  A single
+// GPU-side wait per step covers both hazards: my phase 0 of step n reads the
+// ghost planes the neighbours pushed in step n-1 (RAW), and my pushes in step
+// n overwrite ghost planes they last read in their phase 0 of step n-1 (WAR);
+// both are "neighbours' phase 0 of step n-1 done" = signal word 0 >= n.
+template <typename T> static cudaError_t enqueue_step_push(rafd_room *r, bool prof, int64_t n)
+{
+    cudaError_t e = cudaSuccess;
+    if (n > 0 && (e = ipc_wait_peers(r->ipc, 0, n, r->stream)) != cudaSuccess) return e;
+    int64_t m[2];
+    const int b = r->cur ^ 1;  // u^{n+1}
+    ipc_mirror_deltas(r->ipc, b, r->u[b], (size_t)r->g.plane * sizeof(T), r->g.lnz, &m[0], &m[1]);
+    if ((e = enqueue_phase<T>(r, 0, r->stream, prof, m)) != cudaSuccess) return e;
+    if ((e = ipc_signal(r->ipc_sig + 0, n + 1, r->stream)) != cudaSuccess) return e;  // with a memory fence
+    return enqueue_phase<T>(r, 1, r->stream, prof);
 }
 
 // one NCCL-halo step of this rank
@@ -921,6 +952,10 @@ template <typename T> static int step_t(rafd_room *r, int64_t nsteps)
         if (r->halo) {
             e = enqueue_step_nccl<T>(r, r->profiling);
             if (e == cudaErrorUnknown) return set_err(RAFD_E_NCCL, "%s", halo_last_error());
+            r->launches += kernels_per_phase(r, 0) + kernels_per_phase(r, 1);
+        } else if (r->ipc && r->push) {
+            e = enqueue_step_push<T>(r, r->profiling, r->steps + done);
+            if (e == cudaErrorUnknown) return set_err(RAFD_E_CUDA, "%s", halo_last_error());
             r->launches += kernels_per_phase(r, 0) + kernels_per_phase(r, 1);
         } else if (r->ipc) {
             e = enqueue_step_ipc<T>(r, r->profiling, r->steps + done);
@@ -1068,6 +1103,21 @@ extern "C" int rafd_ipc_connect(rafd_room *r, const uint8_t *lower, const uint8_
     CK(cudaStreamSynchronize(r->stream));
     int rc = ipc_open(&r->ipc, lower, upper, (uint32_t)r->g.pitch);
     if (rc) return set_err(rc, "%s", halo_last_error());
+    return RAFD_OK;
+}
+
+extern "C" int rafd_set_halo_push(rafd_room *r, int32_t on)
+{
+    if (!r) return set_err(RAFD_E_INVAL, "null room");
+    if (!on) {
+        r->push = false;
+        return RAFD_OK;
+    }
+    if (!r->ipc) return set_err(RAFD_E_STATE, "halo push needs an IPC-connected slab (rafd_ipc_connect)");
+    if (r->fused || r->scheme || !r->vplan)
+        return set_err(RAFD_E_STATE, "halo push runs with the two-kernel scheme and the TMA volume kernel");
+    if (r->steps != 0) return set_err(RAFD_E_STATE, "choose the halo transport before the first step");
+    r->push = true;
     return RAFD_OK;
 }
 

@@ -38,6 +38,7 @@ ABI_SYMBOLS = [
     "rafd_set_profiling", "rafd_get_kernel_times", "rafd_launch_count", "rafd_slab_plan",
     "rafd_nccl_unique_id", "rafd_last_error", "rafd_strerror", "rafd_version",
     "rafd_ipc_handle", "rafd_ipc_connect", "rafd_set_step", "rafd_set_temporal_blocking",
+    "rafd_set_halo_push",
 ]
 RAFD_IPC_BLOB_BYTES = 208
 
@@ -115,6 +116,7 @@ def lib():
     L.rafd_nccl_unique_id.argtypes = [P]
     L.rafd_ipc_handle.argtypes = [P, P]
     L.rafd_ipc_connect.argtypes = [P, P, P]
+    L.rafd_set_halo_push.argtypes = [P, I32]
     L.rafd_last_error.restype = C.c_char_p
     L.rafd_strerror.restype = C.c_char_p
     L.rafd_strerror.argtypes = [C.c_int]
@@ -314,6 +316,11 @@ class Room:
         hi = None if upper is None else (C.c_uint8 * RAFD_IPC_BLOB_BYTES).from_buffer_copy(upper)
         _check(lib().rafd_ipc_connect(self.h, None if lo is None else C.addressof(lo),
                                       None if hi is None else C.addressof(hi)))
+
+    def set_halo_push(self, on=True):
+        """rafd_set_halo_push: the edge-phase kernels store the halo into the
+        neighbours' ghost planes (device-initiated) instead of copy pulls."""
+        _check(lib().rafd_set_halo_push(self.h, int(bool(on))))
 
     def launch_count(self):
         return int(lib().rafd_launch_count(self.h))

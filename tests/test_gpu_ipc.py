@@ -2,8 +2,9 @@
 rafd_ipc_connect): p processes on one GPU (the same code path drives peer GPUs
 over NVLink), blobs exchanged with torch.distributed (gloo), halo planes
 pulled by device-to-device copies ordered by GPU-side waits on the
-neighbours' signal words.  The gathered result must equal the undivided room
-bit for bit."""
+neighbours' signal words, or pushed by the edge-phase kernels themselves into
+the neighbours' ghost planes (rafd_set_halo_push, device-initiated).  The
+gathered result must equal the undivided room bit for bit."""
 import math
 import os
 import socket
@@ -42,7 +43,7 @@ def _free_port():
     return p
 
 
-def _worker(rank, world, port, plan, q):
+def _worker(rank, world, port, plan, q, push=False):
     os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
     dist.init_process_group("gloo", rank=rank, world_size=world)
     try:
@@ -57,6 +58,8 @@ def _worker(rank, world, port, plan, q):
         blobs = [None] * world
         dist.all_gather_object(blobs, room.ipc_handle())
         room.ipc_connect(blobs[rank - 1] if rank > 0 else None, blobs[rank + 1] if rank < world - 1 else None)
+        if push:
+            room.set_halo_push(True)
         dist.barrier()
         try:
             room.step(STEPS // 2)
@@ -73,8 +76,9 @@ def _worker(rank, world, port, plan, q):
         dist.destroy_process_group()
 
 
+@pytest.mark.parametrize("push", [False, True])
 @pytest.mark.parametrize("world", [2, 3])
-def test_ipc_slabs_equal_single_room(world):
+def test_ipc_slabs_equal_single_room(world, push):
     from paper_conf_ipps_stoltzfushsld21_b200 import rafd
     mask, mm, beta0, D, E, F, up, uc, src, rcv, sig = _case()
     plan = rafd.rafd_slab_plan(mask, 32, 3, world)
@@ -89,7 +93,7 @@ def test_ipc_slabs_equal_single_room(world):
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
     port = _free_port()
-    procs = [ctx.Process(target=_worker, args=(r, world, port, plan, q)) for r in range(world)]
+    procs = [ctx.Process(target=_worker, args=(r, world, port, plan, q, push)) for r in range(world)]
     for p in procs:
         p.start()
     res = dict((r, (c, pv, rc)) for r, c, pv, rc in (q.get(timeout=120) for _ in range(world)))

@@ -252,3 +252,6 @@ def test_errors():
     s = rafd.Room(mask, LAM, 32, np.array([0.1]), scheme=1)
     with pytest.raises(rafd.RafdError):
         s.set_temporal_blocking(2)
+    with pytest.raises(rafd.RafdError):  # the halo push needs an IPC-connected slab
+        g.set_halo_push(True)
+    g.set_halo_push(False)
