@@ -164,10 +164,10 @@ __global__ void __launch_bounds__(TbGeom<T, TY, SU, SP>::NT, 1)
     using G = TbGeom<T, TY, SU, SP>;
     using KW = typename Vec16<T>::K;
     constexpr int VEC = G::VEC, TX = G::TX, TXO = G::TXO, UROW = G::UROW;
-    extern __shared__ __align__(128) unsigned char smem_raw[];
-    // pointer arithmetic on the shared array (no integer casts) keeps the
-    // accesses in the shared window: LDS/STS with 32-bit addresses
-    unsigned char *base = smem_raw + ((128u - (tb::smem_u32(smem_raw) & 127u)) & 127u);
+    // The dynamic shared window starts 1 KB-aligned (checked below): every slot
+    // is the array plus a compile-time offset (LDS/STS, no runtime alignment).
+    extern __shared__ __align__(1024) unsigned char smem_raw[];
+    unsigned char *const base = smem_raw;
     T *us = (T *)base;                                                  // SU u^n slots
     T *ps = (T *)(base + SU * G::U_BYTES);                              // SP u^{n-1} slots
     uint8_t *ks = base + SU * G::U_BYTES + SP * G::P_BYTES;             // SP K slots
@@ -175,7 +175,9 @@ __global__ void __launch_bounds__(TbGeom<T, TY, SU, SP>::NT, 1)
     uint64_t *bar = (uint64_t *)((unsigned char *)u1s + 2 * G::U1_BYTES);
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
 
+    static_assert((SU & (SU - 1)) == 0 && (SP & (SP - 1)) == 0, "ring sizes are powers of two");
     if (tid == 0) {
+        if (tb::smem_u32(smem_raw) & 127u) __trap();  // TMA destinations need 128-byte alignment
         for (int i = 0; i < SU + SP; i++) tb::mbar_init(&bar[i], 1);
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
@@ -201,27 +203,27 @@ __global__ void __launch_bounds__(TbGeom<T, TY, SU, SP>::NT, 1)
         const int kx = px + k_shift(g);              // K bytes of the region start
         const int kd = kx & 15;                      // its offset in the aligned K box
         auto issue_u = [&](int p) {
-            const int s = (p + 2) % SU;
+            const int s = (p + 2) & (SU - 1);
             tb::mbar_expect_tx(&bar[s], G::U_TX);
             tb::tma_load_3d((unsigned char *)us + s * G::U_BYTES, &umap, &bar[s], ux, uy, p);
         };
         auto issue_pk = [&](int p) {
-            const int s = (p + 1) % SP;
+            const int s = (p + 1) & (SP - 1);
             tb::mbar_expect_tx(&bar[SU + s], G::PK_TX);
             tb::tma_load_3d((unsigned char *)ps + s * G::P_BYTES, &pmap, &bar[SU + s], px, py, p);
             tb::tma_load_3d(ks + s * G::K_BYTES, &kmap, &bar[SU + s], kx - kd, py, p);
         };
         auto wait_u = [&](int p) {
-            const int s = (p + 2) % SU;
+            const int s = (p + 2) & (SU - 1);
             tb::mbar_wait(&bar[s], (uph >> s) & 1);
             uph ^= 1u << s;
         };
         auto wait_pk = [&](int p) {
-            const int s = (p + 1) % SP;
+            const int s = (p + 1) & (SP - 1);
             tb::mbar_wait(&bar[SU + s], (pph >> s) & 1);
             pph ^= 1u << s;
         };
-        auto uslot = [&](int p) -> const T * { return us + ((p + 2) % SU) * (G::U_BYTES / (int)sizeof(T)); };
+        auto uslot = [&](int p) -> const T * { return us + ((p + 2) & (SU - 1)) * (G::U_BYTES / (int)sizeof(T)); };
         // u^n planes pa-2 .. pb+1, u^{n-1}/K planes pa-1 .. pb
         __syncthreads();  // the previous unit is done with every slot
         if (tid == 0) {
@@ -256,8 +258,8 @@ __global__ void __launch_bounds__(TbGeom<T, TY, SU, SP>::NT, 1)
             wait_u(q + 1);
             wait_pk(q);
             const T *uq = uslot(q), *uqp = uslot(q + 1);
-            const T *pq = ps + ((q + 1) % SP) * (G::P_BYTES / (int)sizeof(T));
-            const uint8_t *kq = ks + ((q + 1) % SP) * G::K_BYTES;
+            const T *pq = ps + ((q + 1) & (SP - 1)) * (G::P_BYTES / (int)sizeof(T));
+            const uint8_t *kq = ks + ((q + 1) & (SP - 1)) * G::K_BYTES;
             T *u1w = u1s + (q & 1) * (G::U1_BYTES / (int)sizeof(T));
             T o1p[2][VEC], unp[2][VEC];
             KW kqv[2];
@@ -444,7 +446,7 @@ static bool tb_map(CUtensorMap *m, CUtensorMapDataType dt, size_t esize, void *b
               CU_TENSOR_MAP_L2_PROMOTION_L2_128B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
 }
 
-static constexpr int kTbTY = 32, kTbSU = 4, kTbSP = 3;
+static constexpr int kTbTY = 32, kTbSU = 4, kTbSP = 4;
 
 struct TwoStepPlan {
     CUtensorMap umap[4], pmap[4], kmap;

@@ -15,6 +15,8 @@ import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.path.join(_HERE, "librafd.so")
+# A/B experiments: RAFD_LIB points the binding at another build of the same ABI
+LIB_PATH = os.environ.get("RAFD_LIB", LIB_PATH)
 
 RAFD_OK = 0
 RAFD_E_INVAL = -1
