@@ -186,8 +186,14 @@ int rafd_step(rafd_room *r, int64_t nsteps);
  * (same expressions, same order).  Allocates a second pair of field buffers
  * (the two steps are written out of place) and the shell list; an odd step
  * count ends with one single step.  1 switches back (buffers are kept).
- * Errors: INVAL (not 1 or 2), STATE (a z slab, a fused or single-kernel
- * scheme, or the v0 kernel), NOMEM, CUDA. */
+ * A z slab (any transport) runs the double step edge planes first: u^{n+1}
+ * of its first / last owned plane with the single-step kernel, their exchange
+ * overlapped with the two-step kernel over the interior planes, then u^{n+2}
+ * of the edge planes from the exchanged u^{n+1}, a second exchange overlapped
+ * with the interior shell (one plane per neighbour per step, as single steps).
+ * Every slab of a room must use the same setting.  Errors: INVAL (not 1 or
+ * 2), STATE (a fused or single-kernel scheme, the v0 kernel, an IPC slab
+ * already connected to neighbours that exported two buffers), NOMEM, CUDA. */
 int rafd_set_temporal_blocking(rafd_room *r, int32_t steps_per_sweep);
 
 /* Step the n slabs of one room held by this process (created with nranks = n,
@@ -200,15 +206,18 @@ int rafd_step_group(rafd_room **rooms, int32_t n, int64_t nsteps);
 
 /* Cross-process slabs without NCCL: a slab created with
  * nranks > 1 and nccl_id = NULL exports a RAFD_IPC_BLOB_BYTES blob (CUDA IPC
- * handles of its two field buffers and its two 64-bit signal words, plus its
- * plane count and pitch); the caller exchanges blobs (e.g. torch.distributed
- * all_gather_object) and connects each slab to its neighbours' blobs (NULL at
- * the room's ends).  Afterwards rafd_step runs the edge-first step with the
- * halo planes pulled by device-to-device (peer) copies, ordered by GPU-side
- * stream waits on the neighbours' signal words -- no host round trip, no NCCL.
- * Neighbours may be on the same GPU or on peer GPUs (NVLink).  All slabs must
- * step the same number of times.  Errors: STATE, INVAL, CUDA. */
-#define RAFD_IPC_BLOB_BYTES 208
+ * handles of its field buffers -- two, or four once temporal blocking is on --
+ * and of its signal words, plus its plane count and pitch); the caller
+ * exchanges blobs (e.g. torch.distributed all_gather_object) and connects each
+ * slab to its neighbours' blobs (NULL at the room's ends).  Afterwards
+ * rafd_step runs the edge-first step with the halo planes pulled by
+ * device-to-device (peer) copies, ordered by GPU-side stream waits on the
+ * neighbours' signal words -- no host round trip, no NCCL.  Neighbours may be
+ * on the same GPU or on peer GPUs (NVLink).  All slabs must step the same
+ * number of times with the same steps_per_sweep; with temporal blocking every
+ * slab calls rafd_set_temporal_blocking(r, 2) BEFORE rafd_ipc_handle (the blob
+ * then carries the second buffer pair).  Errors: STATE, INVAL, CUDA. */
+#define RAFD_IPC_BLOB_BYTES 352
 int rafd_ipc_handle(rafd_room *r, uint8_t *blob);
 int rafd_ipc_connect(rafd_room *r, const uint8_t *lower, const uint8_t *upper);
 

@@ -4,6 +4,7 @@
 #include <string.h>
 
 #include <string>
+#include <algorithm>
 
 #include "../../include/rafd.h"
 #include "halo.h"
@@ -149,7 +150,8 @@ cudaError_t halo_exchange(Halo *h, void *buf, size_t plane_bytes, int lnz, cudaS
 namespace rafd {
 
 struct IpcPeer {
-    void *u[2] = {nullptr, nullptr};
+    void *u[4] = {nullptr, nullptr, nullptr, nullptr};
+    int nbuf = 0;
     int64_t *sig = nullptr;
     bool open = false;
     int lnz = 0;
@@ -189,35 +191,40 @@ static StreamMemOps &memops()
     return m;
 }
 
-int ipc_make_blob(void *u0, void *u1, int64_t *sig, int device, int lnz, uint32_t pitch, uint8_t *blob)
+int ipc_make_blob(void *const u[4], int64_t *sig, int device, int lnz, uint32_t pitch, uint8_t *blob)
 {
-    cudaIpcMemHandle_t h[3];
-    void *p[3] = {u0, u1, sig};
-    for (int k = 0; k < 3; k++) {
-        cudaError_t e = cudaIpcGetMemHandle(&h[k], p[k]);
+    memset(blob, 0, kIpcBlobBytes);
+    const int nbuf = (u[2] && u[3]) ? 4 : 2;
+    void *p[5] = {u[0], u[1], nbuf == 4 ? u[2] : nullptr, nbuf == 4 ? u[3] : nullptr, sig};
+    for (int k = 0; k < 5; k++) {
+        if (!p[k]) continue;
+        cudaIpcMemHandle_t h;
+        cudaError_t e = cudaIpcGetMemHandle(&h, p[k]);
         if (e != cudaSuccess) {
             h_err = std::string("cudaIpcGetMemHandle: ") + cudaGetErrorString(e);
             return RAFD_E_CUDA;
         }
-        memcpy(blob + 64 * k, &h[k], 64);
+        memcpy(blob + 64 * k, &h, 64);
     }
-    uint32_t tail[4] = {kMagic, (uint32_t)device, (uint32_t)lnz, pitch};
-    memcpy(blob + 192, tail, 16);
+    uint32_t tail[8] = {kMagic, (uint32_t)device, (uint32_t)lnz, pitch, (uint32_t)nbuf, 0, 0, 0};
+    memcpy(blob + 320, tail, 32);
     return RAFD_OK;
 }
 
 static int open_peer(IpcPeer &pe, const uint8_t *blob)
 {
-    uint32_t tail[4];
-    memcpy(tail, blob + 192, 16);
+    uint32_t tail[8];
+    memcpy(tail, blob + 320, 32);
     if (tail[0] != kMagic) {
         h_err = "not a rafd IPC blob";
         return RAFD_E_INVAL;
     }
     pe.lnz = (int)tail[2];
     pe.pitch = tail[3];
-    void **dst[3] = {&pe.u[0], &pe.u[1], (void **)&pe.sig};
-    for (int k = 0; k < 3; k++) {
+    pe.nbuf = (int)tail[4];
+    void **dst[5] = {&pe.u[0], &pe.u[1], &pe.u[2], &pe.u[3], (void **)&pe.sig};
+    for (int k = 0; k < 5; k++) {
+        if (k >= pe.nbuf && k < 4) continue;
         cudaIpcMemHandle_t h;
         memcpy(&h, blob + 64 * k, 64);
         cudaError_t e = cudaIpcOpenMemHandle(dst[k], h, cudaIpcMemLazyEnablePeerAccess);
@@ -230,13 +237,21 @@ static int open_peer(IpcPeer &pe, const uint8_t *blob)
     return RAFD_OK;
 }
 
+int ipc_peer_buffers(const HaloIpc *h)
+{
+    int n = 4;
+    for (const IpcPeer *pe : {&h->lo, &h->hi})
+        if (pe->open) n = std::min(n, pe->nbuf);
+    return n;
+}
+
 int ipc_open(HaloIpc **out, const uint8_t *lower, const uint8_t *upper, uint32_t pitch)
 {
     *out = nullptr;
     for (const uint8_t *b : {lower, upper}) {
         if (!b) continue;
-        uint32_t tail[4];
-        memcpy(tail, b + 192, 16);
+        uint32_t tail[8];
+        memcpy(tail, b + 320, 32);
         if (tail[0] != kMagic || tail[3] != pitch) {
             h_err = "IPC blob is not a slab of the same room (magic / pitch mismatch)";
             return RAFD_E_INVAL;
@@ -260,7 +275,7 @@ void ipc_close(HaloIpc *h)
     if (!h) return;
     for (IpcPeer *pe : {&h->lo, &h->hi}) {
         if (!pe->open) continue;
-        for (int k = 0; k < 2; k++)
+        for (int k = 0; k < 4; k++)
             if (pe->u[k]) cudaIpcCloseMemHandle(pe->u[k]);
         if (pe->sig) cudaIpcCloseMemHandle(pe->sig);
     }

@@ -28,9 +28,13 @@ const char *halo_last_error();
 // word 1 = "my copies out of my neighbours' buffers for step n done" (n+1).
 namespace rafd {
 struct HaloIpc;
-constexpr int kIpcBlobBytes = 3 * 64 + 16;
-// blob of this rank: IPC handles of u0, u1, sig + (magic, device, lnz, pitch)
-int ipc_make_blob(void *u0, void *u1, int64_t *sig, int device, int lnz, uint32_t pitch, uint8_t *blob);
+constexpr int kIpcBlobBytes = 5 * 64 + 32;
+// blob of this rank: IPC handles of u[0..3] (u[2], u[3] -- the second pair of
+// temporal blocking -- may be null: nbuf = 2) and sig, then (magic, device,
+// lnz, pitch, nbuf)
+int ipc_make_blob(void *const u[4], int64_t *sig, int device, int lnz, uint32_t pitch, uint8_t *blob);
+// number of field buffers every connected neighbour exported (2 or 4)
+int ipc_peer_buffers(const HaloIpc *h);
 int ipc_open(HaloIpc **out, const uint8_t *lower, const uint8_t *upper, uint32_t pitch);
 void ipc_close(HaloIpc *h);
 // per-step pieces (stream-ordered)

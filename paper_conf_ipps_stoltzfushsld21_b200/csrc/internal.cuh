@@ -88,12 +88,13 @@ template <typename T> struct FusedArgs {
 
 // plan == nullptr selects the one-thread-per-voxel v0 kernel (A/B reference);
 // fa->scheme != 0 selects a single-kernel scheme (then no boundary kernel runs);
-// cur_idx = which of the two field buffers holds u^n (selects the TMA maps);
+// cur_idx = which field buffer holds u^n, prev_idx u^{n-1} (default cur_idx ^ 1,
+// in place; selects the TMA maps);
 // fa != nullptr (and a fused plan) applies the boundary update in the same pass.
 template <typename T>
 cudaError_t launch_volume(const Grid &g, const T *cur, T *nxt, const uint8_t *K, double lambda,
                           int z_lo, int z_hi, cudaStream_t s, const void *plan, int cur_idx,
-                          const FusedArgs<T> *fa = nullptr);
+                          const FusedArgs<T> *fa = nullptr, int prev_idx = -1);
 cudaError_t volume_plan_fuse(void *plan, const Grid &g, const uint8_t *K, int64_t Nb, cudaStream_t s);
 bool volume_plan_fused(const void *plan);
 cudaError_t volume_plan_occupancy(void *plan, const Grid &g, const uint8_t *K, cudaStream_t s);
@@ -110,10 +111,12 @@ void twostep_plan_destroy(void *plan);
 cudaError_t twostep_set_source(void *plan, int64_t pos, const Grid &g);
 template <typename T>
 cudaError_t launch_volume2(const void *plan, const Grid &g, int cur_buf, int prev_buf, T *out1, T *out2,
-                           double lambda, cudaStream_t s);
+                           double lambda, cudaStream_t s, int z_lo = 0, int z_hi = -1);
+// interior: only the local planes [1, lnz-1) of a z slab (its edge planes are
+// recomputed whole by the single-step kernel after the halo exchange)
 template <typename T>
 cudaError_t launch_shell(const void *plan, const Grid &g, const T *u1, const T *u0, const uint8_t *K, T *out,
-                         double lambda, cudaStream_t s);
+                         double lambda, cudaStream_t s, bool interior = false);
 template <typename T>
 cudaError_t launch_boundary(int MB, bool idx64, const void *bpos, const uint8_t *Kb,
                             const uint8_t *matb, int64_t i_lo, int64_t i_hi, int64_t Nb, T *unext,

@@ -779,20 +779,10 @@ template <typename T>
 static cudaError_t enqueue_phase(rafd_room *r, int phase, cudaStream_t s, bool prof, const int64_t *mirror = nullptr)
 {
     const Grid &g = r->g;
-    const int lnz = g.lnz, cur = r->cur;
-    T *uc = (T *)r->u[cur];
-    T *un = (T *)r->u[cur ^ 1];
-    auto timed = [&](int kind, auto fn) -> cudaError_t {
-        if (!prof) return fn();
-        cudaEvent_t a, b;
-        cudaEventCreate(&a);
-        cudaEventCreate(&b);
-        cudaEventRecord(a, s);
-        cudaError_t e = fn();
-        cudaEventRecord(b, s);
-        r->evs.push_back({kind, a, b});
-        return e;
-    };
+    const int lnz = g.lnz, cur = r->cur, pc = r->pair + r->cur;
+    T *uc = (T *)r->u[pc];
+    T *un = (T *)r->u[pc ^ 1];
+    auto timed = [&](int kind, auto fn) -> cudaError_t { return timed_launch(r, s, prof, kind, fn); };
     const FusedArgs<T> fa = fused_args<T>(r);
     // mirrors of the first owned plane (to the lower neighbour) and the last (to the upper one)
     const int64_t m_lo = mirror ? mirror[0] : 0, m_hi = mirror ? mirror[1] : 0;
@@ -802,7 +792,7 @@ static cudaError_t enqueue_phase(rafd_room *r, int phase, cudaStream_t s, bool p
         f.mirror[0] = m0;
         f.mirror[1] = m1;
         return timed(0, [&] {
-            return launch_volume<T>(g, uc, un, r->K, r->lambda, zl, zh, s, r->vplan, cur,
+            return launch_volume<T>(g, uc, un, r->K, r->lambda, zl, zh, s, r->vplan, pc,
                                     (r->fused || r->scheme || m0 || m1) ? &f : nullptr);
         });
     };
@@ -846,57 +836,152 @@ static int kernels_per_phase(const rafd_room *r, int phase)
     return (lnz > 2 ? 1 : 0) + nbk * (lnz > 2 && r->n_last_start > r->n_first_plane ? 1 : 0) + 1;
 }
 
-// one IPC-halo step of this rank (step index n since creation)
-template <typename T> static cudaError_t enqueue_step_ipc(rafd_room *r, bool prof, int64_t n)
+// ---- slab double step under temporal blocking (twostep.cu), from the state
+// (pair, cur): A = u^{n-1}, B = u^n -> C = u^{n+1}, D = u^{n+2} in the other
+// pair.  The two-step kernel needs u^n one plane beyond the planes it
+// advances, and u^{n+1} of the edge planes is final only after the
+// neighbours' boundary nodes and source of step n+1 -- so a slab runs:
+//   ph 0 (E1): u^{n+1} of the first / last owned plane with the single-step
+//              kernel (B, A -> C), their boundary nodes (u_b slot cur), the
+//              source if it lies there; then C's edge planes are exchanged
+//   ph 1 (I1): the two-step kernel over the interior planes [1, lnz-1) (B, A
+//              -> C, D; it recomputes u^{n+1} of the edge planes for itself,
+//              unstored), their boundary nodes, the source, the receivers
+//   ph 2 (E2): after the exchange, u^{n+2} of the edge planes (C, B -> D),
+//              their boundary nodes (slot cur^1), the source; D's edge planes
+//              are exchanged
+//   ph 3 (I2): the shell of the interior planes (C, B -> D), their boundary
+//              nodes, the source, the receivers.
+// Every value is the single-step expression on the same operands: bitwise
+// the undivided room.  One plane per neighbour per step is exchanged, as with
+// single steps; the first exchange hides behind the two-step kernel.
+template <typename T>
+static cudaError_t enqueue_tb_phase(rafd_room *r, int ph, cudaStream_t s, bool prof, const int64_t *mirror = nullptr)
 {
+    const Grid &g = r->g;
+    const int lnz = g.lnz, pair = r->pair, cur = r->cur;
+    const int bA = pair + (cur ^ 1), bB = pair + cur, bC = (pair ^ 2) + (cur ^ 1), bD = (pair ^ 2) + cur;
+    const bool second = ph >= 2;
+    const int bu = second ? bC : bB, bp = second ? bB : bA, bo = second ? bD : bC;
+    T *out = (T *)r->u[bo];
+    T *ub = ub_slot<T>(r, second ? cur ^ 1 : cur);
+    auto timed = [&](int kind, auto fn) -> cudaError_t { return timed_launch(r, s, prof, kind, fn); };
+    const int64_t m_lo = mirror ? mirror[0] : 0, m_hi = mirror ? mirror[1] : 0;
+    const int64_t mf0 = m_lo, mf1 = lnz == 1 ? m_hi : 0;
+    auto vol = [&](int zl, int zh, int64_t m0, int64_t m1) {
+        FusedArgs<T> f = fused_args<T>(r);
+        f.mirror[0] = m0;
+        f.mirror[1] = m1;
+        return timed(0, [&] {
+            return launch_volume<T>(g, (const T *)r->u[bu], out, r->K, r->lambda, zl, zh, s, r->vplan, bu,
+                                    (m0 || m1) ? &f : nullptr, bp);
+        });
+    };
+    auto bnd = [&](int64_t lo, int64_t hi, int64_t m0, int64_t m1) -> cudaError_t {
+        if (hi <= lo) return cudaSuccess;
+        return timed(1, [&] {
+            return launch_boundary<T>(r->MB, r->idx64, r->bpos, r->Kb, r->matb, lo, hi, r->nb, out, ub, (T *)r->gst,
+                                      (T *)r->vst, (const T *)r->tab, r->M, r->lambda, s, m0, m1);
+        });
+    };
+    const int zs = r->src_z >= 0 ? r->src_z - r->z0 : -1;
+    const bool src_edge = zs == 0 || zs == lnz - 1;
     cudaError_t e = cudaSuccess;
-    if (n > 0 && (e = ipc_wait_peers(r->ipc, 1, n, r->stream)) != cudaSuccess) return e;  // WAR on my edge planes
-    if ((e = enqueue_phase<T>(r, 0, r->stream, prof)) != cudaSuccess) return e;
-    if ((e = ipc_signal(r->ipc_sig + 0, n + 1, r->stream)) != cudaSuccess) return e;
-    if ((e = cudaEventRecord(r->ev_edge, r->stream)) != cudaSuccess) return e;
-    if ((e = cudaStreamWaitEvent(r->comm_stream, r->ev_edge, 0)) != cudaSuccess) return e;
-    if ((e = ipc_wait_peers(r->ipc, 0, n + 1, r->comm_stream)) != cudaSuccess) return e;
-    if ((e = ipc_pull(r->ipc, r->cur ^ 1, r->u[r->cur ^ 1], (size_t)r->g.plane * sizeof(T), r->g.lnz, r->comm_stream)) !=
-        cudaSuccess)
-        return e;
-    if ((e = ipc_signal(r->ipc_sig + 1, n + 1, r->comm_stream)) != cudaSuccess) return e;
-    if ((e = cudaEventRecord(r->ev_halo, r->comm_stream)) != cudaSuccess) return e;
-    if ((e = enqueue_phase<T>(r, 1, r->stream, prof)) != cudaSuccess) return e;
-    return cudaStreamWaitEvent(r->stream, r->ev_halo, 0);
+    if (ph == 0 || ph == 2) {
+        e = vol(0, 1, mf0, mf1);
+        if (e == cudaSuccess && lnz > 1) e = vol(lnz - 1, lnz, m_hi, 0);
+        if (e == cudaSuccess) e = bnd(0, std::min(r->n_first_plane, r->nb), mf0, mf1);
+        if (e == cudaSuccess && lnz > 1) e = bnd(std::max(r->n_last_start, r->n_first_plane), r->nb, m_hi, 0);
+        const int64_t ms0 = zs == 0 ? mf0 : m_hi, ms1 = zs == 0 ? mf1 : 0;
+        if (e == cudaSuccess && src_edge)
+            e = timed(2, [&] { return launch_src_rcv<T>(out, ub, ctl_of<T>(r), s, 1, ms0, ms1); });
+    } else {
+        if (lnz > 2) {
+            if (ph == 1)
+                e = timed(0, [&] {
+                    return launch_volume2<T>(r->tbplan, g, bB, bA, (T *)r->u[bC], (T *)r->u[bD], r->lambda, s, 1,
+                                             lnz - 1);
+                });
+            else
+                e = timed(3, [&] {
+                    return launch_shell<T>(r->tbplan, g, (const T *)r->u[bC], (const T *)r->u[bB], r->K,
+                                           (T *)r->u[bD], r->lambda, s, true);
+                });
+        }
+        if (e == cudaSuccess && lnz > 2) e = bnd(r->n_first_plane, r->n_last_start, 0, 0);
+        if (e == cudaSuccess)
+            e = timed(2, [&] { return launch_src_rcv<T>(out, ub, ctl_of<T>(r), s, src_edge ? 2 : 3); });
+    }
+    return e;
 }
 
-// one IPC step with the halo pushed by the edge-phase kernels themselves
-// (SURVEY §8(f) f2): their stores of the first / last owned plane also go to
-// the neighbours' ghost planes over peer memory, then one signal.  A single
-// GPU-side wait per step covers both hazards: my phase 0 of step n reads the
-// ghost planes the neighbours pushed in step n-1 (RAW), and my pushes in step
-// n overwrite ghost planes they last read in their phase 0 of step n-1 (WAR);
-// both are "neighbours' phase 0 of step n-1 done" = signal word 0 >= n.
-template <typename T> static cudaError_t enqueue_step_push(rafd_room *r, bool prof, int64_t n)
+// the slab phase `ph` of a single step (0, 1) or of a double step (0..3), and
+// the field buffer whose edge planes the exchange after phase ph (even) sends
+static cudaError_t slab_phase(rafd_room *r, bool two, int ph, cudaStream_t s, bool prof, const int64_t *mirror = nullptr)
 {
-    cudaError_t e = cudaSuccess;
-    if (n > 0 && (e = ipc_wait_peers(r->ipc, 0, n, r->stream)) != cudaSuccess) return e;
-    int64_t m[2];
-    const int b = r->cur ^ 1;  // u^{n+1}
-    ipc_mirror_deltas(r->ipc, b, r->u[b], (size_t)r->g.plane * sizeof(T), r->g.lnz, &m[0], &m[1]);
-    if ((e = enqueue_phase<T>(r, 0, r->stream, prof, m)) != cudaSuccess) return e;
-    if ((e = ipc_signal(r->ipc_sig + 0, n + 1, r->stream)) != cudaSuccess) return e;  // with a memory fence
-    return enqueue_phase<T>(r, 1, r->stream, prof);
+    if (two)
+        return r->prec == 32 ? enqueue_tb_phase<float>(r, ph, s, prof, mirror)
+                             : enqueue_tb_phase<double>(r, ph, s, prof, mirror);
+    return r->prec == 32 ? enqueue_phase<float>(r, ph, s, prof, mirror) : enqueue_phase<double>(r, ph, s, prof, mirror);
+}
+static int exchange_buf(const rafd_room *r, bool two, int ph)
+{
+    if (!two) return r->pair + (r->cur ^ 1);
+    return ph < 2 ? (r->pair ^ 2) + (r->cur ^ 1) : (r->pair ^ 2) + r->cur;
 }
 
-// one NCCL-halo step of this rank
-template <typename T> static cudaError_t enqueue_step_nccl(rafd_room *r, bool prof)
+// One step (two = false) or double step (two = true) of a z slab with its
+// halo transport; n = steps taken so far (the IPC signal words count steps:
+// exactly one exchange per step in both modes).
+//  * NCCL: after the edge phase, ncclSend/ncclRecv of the edge planes on
+//    comm_stream, overlapped with the interior phase; the next edge phase
+//    waits for it.
+//  * IPC pull: the edge phase publishes word 0 = m+1; comm_stream waits for
+//    the neighbours' word 0, copies their edge planes into my ghost planes
+//    (peer copies) and publishes word 1 = m+1; an edge phase first waits for
+//    the neighbours' word 1 >= m (WAR: they finished copying out of my
+//    buffers).
+//  * IPC push: the edge-phase kernels also store their
+//    planes into the neighbours' ghost planes over peer memory, then one
+//    fenced signal word 0 = m+1; the edge phase of step m first waits for the
+//    neighbours' word 0 >= m, which orders both the ghost reads (RAW) and the
+//    next pushes (WAR: a ghost plane is last read in the edge phase -- or the
+//    two-step kernel right after it -- of an earlier step).
+static cudaError_t slab_step(rafd_room *r, bool two, bool prof, int64_t n)
 {
-    cudaError_t e = enqueue_phase<T>(r, 0, r->stream, prof);
-    if (e != cudaSuccess) return e;
-    if ((e = cudaEventRecord(r->ev_edge, r->stream)) != cudaSuccess) return e;
-    if ((e = cudaStreamWaitEvent(r->comm_stream, r->ev_edge, 0)) != cudaSuccess) return e;
-    e = halo_exchange(r->halo, r->u[r->cur ^ 1], (size_t)r->g.plane * sizeof(T), r->g.lnz, r->comm_stream);
-    if (e != cudaSuccess) return e;
-    if ((e = cudaEventRecord(r->ev_halo, r->comm_stream)) != cudaSuccess) return e;
-    e = enqueue_phase<T>(r, 1, r->stream, prof);
-    if (e != cudaSuccess) return e;
-    return cudaStreamWaitEvent(r->stream, r->ev_halo, 0);  // ghost planes ready for the next step
+    cudaError_t e = cudaSuccess;
+    const size_t pb = (size_t)r->g.plane * r->s;
+    const int lnz = r->g.lnz;
+    for (int h = 0; h < (two ? 2 : 1); h++) {
+        const int64_t m = n + h;
+        const int pe = two ? 2 * h : 0, pi = pe + 1;
+        const int xb = exchange_buf(r, two, pe);
+        if (r->ipc && r->push) {
+            if (m > 0 && (e = ipc_wait_peers(r->ipc, 0, m, r->stream)) != cudaSuccess) return e;
+            int64_t mr[2];
+            ipc_mirror_deltas(r->ipc, xb, r->u[xb], pb, lnz, &mr[0], &mr[1]);
+            if ((e = slab_phase(r, two, pe, r->stream, prof, mr)) != cudaSuccess) return e;
+            if ((e = ipc_signal(r->ipc_sig + 0, m + 1, r->stream)) != cudaSuccess) return e;  // with a memory fence
+            if ((e = slab_phase(r, two, pi, r->stream, prof)) != cudaSuccess) return e;
+            continue;
+        }
+        if (r->ipc && m > 0 && (e = ipc_wait_peers(r->ipc, 1, m, r->stream)) != cudaSuccess) return e;
+        if ((e = slab_phase(r, two, pe, r->stream, prof)) != cudaSuccess) return e;
+        if (r->ipc && (e = ipc_signal(r->ipc_sig + 0, m + 1, r->stream)) != cudaSuccess) return e;
+        if ((e = cudaEventRecord(r->ev_edge, r->stream)) != cudaSuccess) return e;
+        if ((e = cudaStreamWaitEvent(r->comm_stream, r->ev_edge, 0)) != cudaSuccess) return e;
+        if (r->ipc) {
+            if ((e = ipc_wait_peers(r->ipc, 0, m + 1, r->comm_stream)) != cudaSuccess) return e;
+            if ((e = ipc_pull(r->ipc, xb, r->u[xb], pb, lnz, r->comm_stream)) != cudaSuccess) return e;
+            if ((e = ipc_signal(r->ipc_sig + 1, m + 1, r->comm_stream)) != cudaSuccess) return e;
+        } else {
+            if ((e = halo_exchange(r->halo, r->u[xb], pb, lnz, r->comm_stream)) != cudaSuccess) return e;
+        }
+        if ((e = cudaEventRecord(r->ev_halo, r->comm_stream)) != cudaSuccess) return e;
+        if ((e = slab_phase(r, two, pi, r->stream, prof)) != cudaSuccess) return e;
+        if ((e = cudaStreamWaitEvent(r->stream, r->ev_halo, 0)) != cudaSuccess) return e;  // ghost planes ready
+    }
+    return e;
 }
 
 static int kernels_per_step(const rafd_room *r) { return 2 + (r->nb > 0 && !r->fused && !r->scheme ? 1 : 0); }
@@ -940,32 +1025,30 @@ template <typename T> static int step_t(rafd_room *r, int64_t nsteps)
         r->launches += r->tb == 2 ? (int64_t)kernels_per_double_step(r) * (rafd_room::G / 2) : (int64_t)kps * rafd_room::G;
     }
     // temporal blocking: double steps, an odd last step runs single
+    const bool slab = r->halo || r->ipc;
+    auto slab_err = [&](cudaError_t e) {
+        if (e == cudaErrorUnknown) return set_err(r->halo ? RAFD_E_NCCL : RAFD_E_CUDA, "%s", halo_last_error());
+        return set_err(RAFD_E_CUDA, "step: %s", cudaGetErrorString(e));
+    };
+    const int64_t kslab = slab ? kernels_per_phase(r, 0) + kernels_per_phase(r, 1) : 0;
     while (r->tb == 2 && nsteps - done >= 2) {
-        cudaError_t e = enqueue_step2<T>(r, r->pair, r->cur, r->stream, r->profiling);
-        if (e != cudaSuccess) return set_err(RAFD_E_CUDA, "step: %s", cudaGetErrorString(e));
-        r->launches += kernels_per_double_step(r);
+        cudaError_t e = slab ? slab_step(r, true, r->profiling, r->steps + done)
+                             : enqueue_step2<T>(r, r->pair, r->cur, r->stream, r->profiling);
+        if (e != cudaSuccess) return slab ? slab_err(e) : set_err(RAFD_E_CUDA, "step: %s", cudaGetErrorString(e));
+        r->launches += slab ? 2 * kslab : kernels_per_double_step(r);
         r->pair ^= 2;
         done += 2;
     }
     for (; done < nsteps; done++) {
-        cudaError_t e;
-        if (r->halo) {
-            e = enqueue_step_nccl<T>(r, r->profiling);
-            if (e == cudaErrorUnknown) return set_err(RAFD_E_NCCL, "%s", halo_last_error());
-            r->launches += kernels_per_phase(r, 0) + kernels_per_phase(r, 1);
-        } else if (r->ipc && r->push) {
-            e = enqueue_step_push<T>(r, r->profiling, r->steps + done);
-            if (e == cudaErrorUnknown) return set_err(RAFD_E_CUDA, "%s", halo_last_error());
-            r->launches += kernels_per_phase(r, 0) + kernels_per_phase(r, 1);
-        } else if (r->ipc) {
-            e = enqueue_step_ipc<T>(r, r->profiling, r->steps + done);
-            if (e == cudaErrorUnknown) return set_err(RAFD_E_CUDA, "%s", halo_last_error());
-            r->launches += kernels_per_phase(r, 0) + kernels_per_phase(r, 1);
+        if (slab) {
+            cudaError_t e = slab_step(r, false, r->profiling, r->steps + done);
+            if (e != cudaSuccess) return slab_err(e);
+            r->launches += kslab;
         } else {
-            e = enqueue_step<T>(r, r->pair, r->cur, r->stream, r->profiling);
+            cudaError_t e = enqueue_step<T>(r, r->pair, r->cur, r->stream, r->profiling);
+            if (e != cudaSuccess) return set_err(RAFD_E_CUDA, "step: %s", cudaGetErrorString(e));
             r->launches += kps;
         }
-        if (e != cudaSuccess) return set_err(RAFD_E_CUDA, "step: %s", cudaGetErrorString(e));
         r->cur ^= 1;
     }
     r->steps += nsteps;
@@ -994,54 +1077,60 @@ template <typename T> static int step_group_t(rafd_room **rs, int n, int64_t nst
         int rc = ensure_rec<T>(rs[k], nsteps);
         if (rc) return rc;
     }
-    for (int64_t st = 0; st < nsteps; st++) {
-        // phase 0 of every slab (after the neighbours finished copying out of
-        // the buffer this step overwrites... they read our u^{n}, which we
-        // overwrite one step later; waiting here is sufficient)
-        for (int k = 0; k < n; k++) {
-            rafd_room *r = rs[k];
-            CK(cudaSetDevice(r->device));
-            if (st > 0) {
+    const bool tb2 = rs[0]->tb == 2;  // temporal blocking: double steps (enqueue_tb_phase), an odd last one single
+    for (int64_t done = 0; done < nsteps;) {
+        const bool two = tb2 && nsteps - done >= 2;
+        for (int h = 0; h < (two ? 2 : 1); h++) {
+            const int pe = two ? 2 * h : 0;
+            // edge phase of every slab, after the neighbours finished copying
+            // out of its buffers (their previous pulls)
+            for (int k = 0; k < n; k++) {
+                rafd_room *r = rs[k];
+                CK(cudaSetDevice(r->device));
                 if (k > 0) CK(cudaStreamWaitEvent(r->stream, rs[k - 1]->ev_halo, 0));
                 if (k < n - 1) CK(cudaStreamWaitEvent(r->stream, rs[k + 1]->ev_halo, 0));
+                cudaError_t e = slab_phase(r, two, pe, r->stream, r->profiling);
+                if (e != cudaSuccess) return set_err(RAFD_E_CUDA, "step: %s", cudaGetErrorString(e));
+                CK(cudaEventRecord(r->ev_edge, r->stream));
+                r->launches += kernels_per_phase(r, 0);
             }
-            cudaError_t e = enqueue_phase<T>(r, 0, r->stream, r->profiling);
-            if (e != cudaSuccess) return set_err(RAFD_E_CUDA, "step: %s", cudaGetErrorString(e));
-            CK(cudaEventRecord(r->ev_edge, r->stream));
-            r->launches += kernels_per_phase(r, 0);
+            // halo: each slab pulls its ghost planes on its comm stream
+            for (int k = 0; k < n; k++) {
+                rafd_room *r = rs[k];
+                CK(cudaSetDevice(r->device));
+                const size_t pb = (size_t)r->g.plane * sizeof(T);
+                char *mine = (char *)r->u[exchange_buf(r, two, pe)];
+                CK(cudaStreamWaitEvent(r->comm_stream, r->ev_edge, 0));
+                if (k > 0) {
+                    rafd_room *q = rs[k - 1];
+                    CK(cudaStreamWaitEvent(r->comm_stream, q->ev_edge, 0));
+                    const char *src = (const char *)q->u[exchange_buf(q, two, pe)] + (size_t)q->g.lnz * pb;
+                    CK(cudaMemcpyPeerAsync(mine, r->device, src, q->device, pb, r->comm_stream));
+                }
+                if (k < n - 1) {
+                    rafd_room *q = rs[k + 1];
+                    CK(cudaStreamWaitEvent(r->comm_stream, q->ev_edge, 0));
+                    const char *src = (const char *)q->u[exchange_buf(q, two, pe)] + pb;
+                    CK(cudaMemcpyPeerAsync(mine + (size_t)(r->g.lnz + 1) * pb, r->device, src, q->device, pb,
+                                           r->comm_stream));
+                }
+                CK(cudaEventRecord(r->ev_halo, r->comm_stream));
+            }
+            // interior phase overlapped with the copies
+            for (int k = 0; k < n; k++) {
+                rafd_room *r = rs[k];
+                CK(cudaSetDevice(r->device));
+                cudaError_t e = slab_phase(r, two, pe + 1, r->stream, r->profiling);
+                if (e != cudaSuccess) return set_err(RAFD_E_CUDA, "step: %s", cudaGetErrorString(e));
+                CK(cudaStreamWaitEvent(r->stream, r->ev_halo, 0));
+                r->launches += kernels_per_phase(r, 1);
+            }
         }
-        // halo: each slab pulls its ghost planes on its comm stream
         for (int k = 0; k < n; k++) {
-            rafd_room *r = rs[k];
-            CK(cudaSetDevice(r->device));
-            const size_t pb = (size_t)r->g.plane * sizeof(T);
-            char *mine = (char *)r->u[r->cur ^ 1];  // u^{n+1} of this slab
-            CK(cudaStreamWaitEvent(r->comm_stream, r->ev_edge, 0));
-            if (k > 0) {
-                rafd_room *q = rs[k - 1];
-                CK(cudaStreamWaitEvent(r->comm_stream, q->ev_edge, 0));
-                const char *src = (const char *)q->u[q->cur ^ 1] + (size_t)q->g.lnz * pb;
-                CK(cudaMemcpyPeerAsync(mine, r->device, src, q->device, pb, r->comm_stream));
-            }
-            if (k < n - 1) {
-                rafd_room *q = rs[k + 1];
-                CK(cudaStreamWaitEvent(r->comm_stream, q->ev_edge, 0));
-                const char *src = (const char *)q->u[q->cur ^ 1] + pb;
-                CK(cudaMemcpyPeerAsync(mine + (size_t)(r->g.lnz + 1) * pb, r->device, src, q->device, pb,
-                                       r->comm_stream));
-            }
-            CK(cudaEventRecord(r->ev_halo, r->comm_stream));
+            if (two) rs[k]->pair ^= 2;
+            else rs[k]->cur ^= 1;
         }
-        // phase 1 (interior) overlapped with the copies
-        for (int k = 0; k < n; k++) {
-            rafd_room *r = rs[k];
-            CK(cudaSetDevice(r->device));
-            cudaError_t e = enqueue_phase<T>(r, 1, r->stream, r->profiling);
-            if (e != cudaSuccess) return set_err(RAFD_E_CUDA, "step: %s", cudaGetErrorString(e));
-            CK(cudaStreamWaitEvent(r->stream, r->ev_halo, 0));
-            r->launches += kernels_per_phase(r, 1);
-        }
-        for (int k = 0; k < n; k++) rs[k]->cur ^= 1;
+        done += two ? 2 : 1;
     }
     for (int k = 0; k < n; k++) {
         rs[k]->steps += nsteps;
@@ -1060,6 +1149,7 @@ extern "C" int rafd_step_group(rafd_room **rooms, int32_t n, int64_t nsteps)
             return set_err(RAFD_E_STATE, "group member %d is not local slab %d of %d", k, k, n);
         if (r->prec != rooms[0]->prec || r->nx != rooms[0]->nx || r->ny != rooms[0]->ny || r->nz != rooms[0]->nz)
             return set_err(RAFD_E_STATE, "group members are not slabs of one room");
+        if (r->tb != rooms[0]->tb) return set_err(RAFD_E_STATE, "group members differ in steps_per_sweep");
         if (k > 0 && rooms[k - 1]->z1 != r->z0) return set_err(RAFD_E_STATE, "slabs are not contiguous");
     }
     if (nsteps == 0) return RAFD_OK;
@@ -1087,7 +1177,7 @@ extern "C" int rafd_ipc_handle(rafd_room *r, uint8_t *blob)
     if (!r || !blob) return set_err(RAFD_E_INVAL, "bad arguments");
     if (!r->local_slab || !r->ipc_sig) return set_err(RAFD_E_STATE, "IPC handles exist for slabs created without nccl_id");
     CK(cudaSetDevice(r->device));
-    int rc = ipc_make_blob(r->u[0], r->u[1], r->ipc_sig, r->device, r->g.lnz, (uint32_t)r->g.pitch, blob);
+    int rc = ipc_make_blob(r->u, r->ipc_sig, r->device, r->g.lnz, (uint32_t)r->g.pitch, blob);
     if (rc) return set_err(rc, "%s", halo_last_error());
     return RAFD_OK;
 }
@@ -1471,8 +1561,9 @@ extern "C" int rafd_set_temporal_blocking(rafd_room *r, int32_t steps_per_sweep)
     if (steps_per_sweep == r->tb) return RAFD_OK;
     CK(cudaStreamSynchronize(r->stream));
     if (steps_per_sweep == 2) {
-        if (r->nranks > 1 || r->halo || r->ipc || r->local_slab)
-            return set_err(RAFD_E_STATE, "temporal blocking needs a whole room on one GPU (not a z slab)");
+        if (r->ipc && ipc_peer_buffers(r->ipc) < 4)
+            return set_err(RAFD_E_STATE, "IPC slabs enable temporal blocking before rafd_ipc_handle (the neighbours "
+                                         "exported two field buffers)");
         if (r->scheme != 0 || r->fused)
             return set_err(RAFD_E_STATE, "temporal blocking runs the two-kernel scheme (not fused, not Listing 1/6)");
         if (!r->vplan) return set_err(RAFD_E_STATE, "temporal blocking needs the TMA volume kernel (not v0)");

@@ -159,7 +159,7 @@ template <typename T, int TY, int SU, int SP>
 __global__ void __launch_bounds__(TbGeom<T, TY, SU, SP>::NT, 1)
     k_volume2(const __grid_constant__ CUtensorMap umap, const __grid_constant__ CUtensorMap pmap,
               const __grid_constant__ CUtensorMap kmap, T *__restrict__ out1, T *__restrict__ out2, Grid g, T l2,
-              int zchunk, int tiles_x, int tiles_y)
+              int z_lo, int z_hi, int zchunk, int tiles_x, int tiles_y)
 {
     using G = TbGeom<T, TY, SU, SP>;
     using KW = typename Vec16<T>::K;
@@ -185,7 +185,9 @@ __global__ void __launch_bounds__(TbGeom<T, TY, SU, SP>::NT, 1)
     uint32_t uph = 0, pph = 0;
     const uint64_t pol = tb::policy_evict_first();
 
-    const int nz = g.lnz;
+    // stored planes: local [z_lo, z_hi) (a z slab stores its interior planes;
+    // the u^n ghost planes it reads are the neighbours' edge planes)
+    const int nz = z_hi - z_lo;
     const int nchunks = (nz + zchunk - 1) / zchunk;
     const int tiles = tiles_x * tiles_y;
     const int units = nchunks * tiles;
@@ -194,8 +196,8 @@ __global__ void __launch_bounds__(TbGeom<T, TY, SU, SP>::NT, 1)
     for (int unit = blockIdx.x; unit < units; unit += gridDim.x) {
         const int chunk = unit / tiles, t = unit % tiles;
         const int ty = t / tiles_x, tx = t % tiles_x;
-        const int pa = 1 + chunk * zchunk;          // first padded plane stored
-        const int pb = min(1 + nz, pa + zchunk);    // one past the last
+        const int pa = 1 + z_lo + chunk * zchunk;   // first padded plane stored
+        const int pb = min(1 + z_hi, pa + zchunk);  // one past the last
         const int ox = tx * TXO, oy = ty * TY;      // core origin (room coordinates)
         const int ux = g.xo + ox - 2 * VEC;         // u^n box origin (padded x)
         const int uy = oy - 1;                      // padded row of core row -2
@@ -396,16 +398,21 @@ __global__ void k_shell_compact(Grid g, const uint8_t *__restrict__ K, const int
 // u^{n+2} at the shell voxels and the source's 7-point star (src[7], -1 =
 // none), from the final u^{n+1} (u1) and u^n (u0): the volume update in the
 // order of DESIGN.md §4 (same expression as vol_vec).
+// A slab recomputes only its interior planes (padded [zp_lo, zp_hi)): the list
+// is then the sub-range of those planes and star entries elsewhere are skipped
+// (its edge planes are recomputed whole from the exchanged u^{n+1}).
 template <typename T, typename IdxT>
 __global__ void __launch_bounds__(256) k_shell(const IdxT *__restrict__ list, int64_t n, const int64_t *__restrict__ src,
                                                const T *__restrict__ u1, const T *__restrict__ u0,
-                                               const uint8_t *__restrict__ K, T *__restrict__ out, Grid g, T l2)
+                                               const uint8_t *__restrict__ K, T *__restrict__ out, Grid g, T l2,
+                                               int zp_lo, int zp_hi)
 {
     using R = rn<T>;
     const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     if (i >= n + 7) return;
     const int64_t p = i < n ? (int64_t)list[i] : src[i - n];
     if (p < 0) return;
+    if (i >= n && (p < (int64_t)zp_lo * g.plane || p >= (int64_t)zp_hi * g.plane)) return;
     const int nbr = K[p];
     if (nbr == 0) return;
     T s = R::add(u1[p - 1], u1[p + 1]);
@@ -453,6 +460,7 @@ struct TwoStepPlan {
     int tiles_x, tiles_y, grid, smem;
     void *list = nullptr;  // shell positions (uint32 or int64), ascending
     int64_t n_shell = 0;
+    int64_t sh_lo = 0, sh_hi = 0;  // list range of the local planes [1, lnz-1) (slab interior)
     int64_t *src = nullptr;  // [7] the source's star, -1 = none
     bool idx64 = false;
 };
@@ -502,6 +510,9 @@ cudaError_t twostep_plan_create(const Grid &g, void *const u[4], uint8_t *K_allo
     if (e == cudaSuccess) e = exclusive_scan_rows64(cnt, off, rows + 1, tmp, &tb, s);
     int64_t n = 0;
     if (e == cudaSuccess) e = cudaMemcpyAsync(&n, off + rows, 8, cudaMemcpyDeviceToHost, s);
+    if (e == cudaSuccess && g.lnz >= 2) e = cudaMemcpyAsync(&pl->sh_lo, off + g.ny, 8, cudaMemcpyDeviceToHost, s);
+    if (e == cudaSuccess && g.lnz >= 2)
+        e = cudaMemcpyAsync(&pl->sh_hi, off + (int64_t)(g.lnz - 1) * g.ny, 8, cudaMemcpyDeviceToHost, s);
     if (e == cudaSuccess) e = cudaStreamSynchronize(s);
     if (e == cudaSuccess) e = cudaMalloc(&pl->list, (size_t)std::max<int64_t>(n, 1) * (idx64 ? 8 : 4));
     if (e == cudaSuccess && rows > 0 && n > 0) {
@@ -568,44 +579,50 @@ static int tb_choose_zchunk(int nz, int tiles, int grid)
 
 template <typename T>
 cudaError_t launch_volume2(const void *plan, const Grid &g, int cur_buf, int prev_buf, T *out1, T *out2,
-                           double lambda, cudaStream_t s)
+                           double lambda, cudaStream_t s, int z_lo, int z_hi)
 {
     using G = TbGeom<T, kTbTY, kTbSU, kTbSP>;
     const auto *pl = (const TwoStepPlan *)plan;
-    if (g.lnz <= 0) return cudaSuccess;
+    if (z_hi < 0) z_hi = g.lnz;
+    if (z_hi <= z_lo) return cudaSuccess;
     const T l2 = (T)(lambda * lambda);
     const int tiles = pl->tiles_x * pl->tiles_y;
-    const int zc = tb_choose_zchunk(g.lnz, tiles, pl->grid);
-    const long units = (long)tiles * ((g.lnz + zc - 1) / zc);
+    const int zc = tb_choose_zchunk(z_hi - z_lo, tiles, pl->grid);
+    const long units = (long)tiles * ((z_hi - z_lo + zc - 1) / zc);
     const int grid = (int)std::min<long>(pl->grid, units);
     k_volume2<T, kTbTY, kTbSU, kTbSP><<<grid, G::NT, pl->smem, s>>>(pl->umap[cur_buf], pl->pmap[prev_buf], pl->kmap,
-                                                                    out1, out2, g, l2, zc, pl->tiles_x, pl->tiles_y);
+                                                                    out1, out2, g, l2, z_lo, z_hi, zc, pl->tiles_x,
+                                                                    pl->tiles_y);
     return cudaGetLastError();
 }
 
 template <typename T>
 cudaError_t launch_shell(const void *plan, const Grid &g, const T *u1, const T *u0, const uint8_t *K, T *out,
-                         double lambda, cudaStream_t s)
+                         double lambda, cudaStream_t s, bool interior)
 {
     const auto *pl = (const TwoStepPlan *)plan;
     const T l2 = (T)(lambda * lambda);
-    const int64_t n = pl->n_shell + 7;
+    if (interior && g.lnz < 3) return cudaSuccess;
+    const int64_t lo = interior ? pl->sh_lo : 0, cnt = interior ? pl->sh_hi - pl->sh_lo : pl->n_shell;
+    const int zp_lo = interior ? 2 : 1, zp_hi = interior ? g.lnz : g.lnz + 1;
+    const int64_t n = cnt + 7;
     const unsigned blocks = (unsigned)((n + 255) / 256);
     if (pl->idx64)
-        k_shell<T, int64_t><<<blocks, 256, 0, s>>>((const int64_t *)pl->list, pl->n_shell, pl->src, u1, u0, K, out,
-                                                   g, l2);
+        k_shell<T, int64_t><<<blocks, 256, 0, s>>>((const int64_t *)pl->list + lo, cnt, pl->src, u1, u0, K, out, g,
+                                                   l2, zp_lo, zp_hi);
     else
-        k_shell<T, uint32_t><<<blocks, 256, 0, s>>>((const uint32_t *)pl->list, pl->n_shell, pl->src, u1, u0, K, out,
-                                                    g, l2);
+        k_shell<T, uint32_t><<<blocks, 256, 0, s>>>((const uint32_t *)pl->list + lo, cnt, pl->src, u1, u0, K, out, g,
+                                                    l2, zp_lo, zp_hi);
     return cudaGetLastError();
 }
 
 #define RAFD_TB_INST(T)                                                                                            \
     template cudaError_t twostep_plan_create<T>(const Grid &, void *const[4], uint8_t *, const uint8_t *, bool, int, \
                                                 cudaStream_t, void **, int64_t *);                                  \
-    template cudaError_t launch_volume2<T>(const void *, const Grid &, int, int, T *, T *, double, cudaStream_t);   \
+    template cudaError_t launch_volume2<T>(const void *, const Grid &, int, int, T *, T *, double, cudaStream_t,    \
+                                           int, int);                                                               \
     template cudaError_t launch_shell<T>(const void *, const Grid &, const T *, const T *, const uint8_t *, T *,     \
-                                         double, cudaStream_t);
+                                         double, cudaStream_t, bool);
 RAFD_TB_INST(float)
 RAFD_TB_INST(double)
 #undef RAFD_TB_INST

@@ -42,7 +42,7 @@ ABI_SYMBOLS = [
     "rafd_ipc_handle", "rafd_ipc_connect", "rafd_set_step", "rafd_set_temporal_blocking",
     "rafd_set_halo_push",
 ]
-RAFD_IPC_BLOB_BYTES = 208
+RAFD_IPC_BLOB_BYTES = 352
 
 
 class rafd_materials(C.Structure):

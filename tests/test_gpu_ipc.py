@@ -18,7 +18,7 @@ import torch.multiprocessing as mp
 pytestmark = pytest.mark.gpu
 LAM = 1.0 / math.sqrt(3.0)
 DIMS = (40, 34, 30)
-STEPS = 60
+STEPS = 61  # the second call is odd: double steps then one single step
 
 
 def _case():
@@ -43,7 +43,7 @@ def _free_port():
     return p
 
 
-def _worker(rank, world, port, plan, q, push=False):
+def _worker(rank, world, port, plan, q, push=False, tb=1):
     os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
     dist.init_process_group("gloo", rank=rank, world_size=world)
     try:
@@ -55,6 +55,8 @@ def _worker(rank, world, port, plan, q, push=False):
         room.set_state(up, uc)
         room.set_source(src, sig)
         room.set_receivers(rcv)
+        if tb == 2:
+            room.set_temporal_blocking(2)  # before the blob: it carries the second buffer pair
         blobs = [None] * world
         dist.all_gather_object(blobs, room.ipc_handle())
         room.ipc_connect(blobs[rank - 1] if rank > 0 else None, blobs[rank + 1] if rank < world - 1 else None)
@@ -76,9 +78,12 @@ def _worker(rank, world, port, plan, q, push=False):
         dist.destroy_process_group()
 
 
+@pytest.mark.parametrize("tb", [1, 2])
 @pytest.mark.parametrize("push", [False, True])
 @pytest.mark.parametrize("world", [2, 3])
-def test_ipc_slabs_equal_single_room(world, push):
+def test_ipc_slabs_equal_single_room(world, push, tb):
+    """tb = 2: temporal blocking in every slab (edge planes single-step, the
+    two-step kernel over the interior; two exchanges per double step)."""
     from paper_conf_ipps_stoltzfushsld21_b200 import rafd
     mask, mm, beta0, D, E, F, up, uc, src, rcv, sig = _case()
     plan = rafd.rafd_slab_plan(mask, 32, 3, world)
@@ -93,7 +98,7 @@ def test_ipc_slabs_equal_single_room(world, push):
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
     port = _free_port()
-    procs = [ctx.Process(target=_worker, args=(r, world, port, plan, q, push)) for r in range(world)]
+    procs = [ctx.Process(target=_worker, args=(r, world, port, plan, q, push, tb)) for r in range(world)]
     for p in procs:
         p.start()
     res = dict((r, (c, pv, rc)) for r, c, pv, rc in (q.get(timeout=120) for _ in range(world)))
