@@ -208,14 +208,14 @@ def run_rafd(args, rank, world, local_rank):
     room = rafd.Room(mask, LAM, prec, beta0, D, E, F, matmap=mm, device=local_rank,
                      stream=stream.cuda_stream, rank=rank, nranks=world, nccl_id=nccl_id,
                      z_begin=z0, z_end=z1, mask_z0=mz0, dims=(nx, ny, nz))
-    tb = args.tb  # temporal blocking (a slab: edge planes single-step, the interior two-step)
-    if tb == 2:
-        room.set_temporal_blocking(2)  # before the IPC blob: it carries the second buffer pair
+    del mask, mm
+    torch.cuda.empty_cache()
+    # temporal blocking (a slab: edge planes single-step, the interior two-step),
+    # before the IPC blob (it carries the second buffer pair)
+    tb = enable_tb(room, args.tb, world, dev)
     if world > 1 and args.transport in ("ipc", "push"):
         connect_ipc(room, rank, world, push=args.transport == "push")
     t_create = time.perf_counter() - t_c
-    del mask, mm
-    torch.cuda.empty_cache()
     mask_np = None if cfg["shape"] == "box" else I.make_mask(cfg["shape"], nx, ny, nz).numpy()
     room.set_source(I.source_position((nx, ny, nz), mask_np), I.impulse())
     room.set_receivers(I.receiver_positions((nx, ny, nz), mask_np))
@@ -301,9 +301,11 @@ def run_rafd(args, rank, world, local_rank):
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(ms_max / args.steps, 4),
             "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
             "dtype": "f32" if prec == 32 else "f64",
-            "data": "synthetic (seeded box hall, region materials, seeded FD tables, impulse source)",
+            "data": f"synthetic (seeded {cfg['shape']} room, {cfg['rule']} materials, "
+                    + ("seeded FD tables" if cfg['MB'] else "FI admittances from absorption") + ", impulse source)",
             "config": {
-                "workload": f"{args.config}: {nx}x{ny}x{nz} box hall, FD-MM MB={cfg['MB']} M={cfg['M']}, "
+                "workload": f"{args.config}: {nx}x{ny}x{nz} {cfg['shape']} room, "
+                            + (f"FD-MM MB={cfg['MB']}" if cfg['MB'] else "FI-MM") + f" M={cfg['M']}, "
                             f"fp{prec}" + (f", {world} z-slabs" if world > 1 else ""),
                 "room_dims_xyz": [nx, ny, nz], "n_inside": int(n_in_total),
                 "halo_transport": args.transport if world > 1 else None,
@@ -352,6 +354,29 @@ def run_rafd(args, rank, world, local_rank):
     return out
 
 
+def enable_tb(room, want, world, dev):
+    """Two leapfrog steps per sweep when asked for and the second buffer pair
+    fits (C5 fp32 on one GPU needs ~143 GB); every rank must run the same
+    setting, so a NOMEM anywhere falls back to single steps everywhere."""
+    from paper_conf_ipps_stoltzfushsld21_b200 import rafd
+    tb = 1
+    if want == 2:
+        try:
+            room.set_temporal_blocking(2)
+            tb = 2
+        except rafd.RafdError as e:
+            if e.code != rafd.RAFD_E_NOMEM:
+                raise
+            print(f"temporal blocking does not fit ({e}); single steps", file=sys.stderr)
+    if world > 1:
+        t = torch.tensor([tb], dtype=torch.int32, device=dev)
+        torch.distributed.all_reduce(t, op=torch.distributed.ReduceOp.MIN)
+        if int(t[0]) != tb:
+            room.set_temporal_blocking(1)
+            tb = 1
+    return tb
+
+
 def run_e2e(args, cfg, prec, beta0, D, E, F, rank, world, local_rank, plan, multi):
     """End to end through the public API with HOST buffers: create the room from
     pinned host mask/matmap (H2D + on-device classification), set source and
@@ -385,9 +410,7 @@ def run_e2e(args, cfg, prec, beta0, D, E, F, rank, world, local_rank, plan, mult
     room = rafd.Room(mask_h.numpy(), LAM, prec, beta0, D, E, F, matmap=mm_h.numpy(), device=local_rank,
                      rank=rank, nranks=world, nccl_id=nccl_id, z_begin=z0, z_end=z1, mask_z0=mz0,
                      dims=(nx, ny, nz))
-    tb = args.tb
-    if tb == 2:
-        room.set_temporal_blocking(2)
+    tb = enable_tb(room, args.tb, world, torch.device("cuda", local_rank))
     if ipc:
         connect_ipc(room, rank, world, push=args.transport == "push")
     room.set_source(I.source_position((nx, ny, nz), mask_np), sig)

@@ -559,12 +559,26 @@ cudaError_t twostep_set_source(void *plan, int64_t pos, const Grid &g)
     return cudaMemcpy(pl->src, h, sizeof h, cudaMemcpyHostToDevice);
 }
 
+// Cap on the planes one unit marches (RAFD_TB_ZCHUNK_MAX, default 0 = none):
+// long marches let the CTAs drift apart in z.
+static int tb_zchunk_cap()
+{
+    static int v = -1;
+    if (v < 0) {
+        const char *e = getenv("RAFD_TB_ZCHUNK_MAX");
+        v = e ? std::max(0, atoi(e)) : 0;
+    }
+    return v;
+}
+
 static int tb_choose_zchunk(int nz, int tiles, int grid)
 {
     long best = -1;
-    int best_c = nz;
+    const int cap = tb_zchunk_cap();
+    int best_c = cap ? std::min(nz, cap) : nz;
     for (int n = 1; n <= nz; n++) {
         const int c = (nz + n - 1) / n;
+        if (cap && c > cap) continue;
         const long units = (long)tiles * ((nz + c - 1) / c);
         const long rounds = (units + grid - 1) / grid;
         const long cost = rounds * (c + 4);  // +4: the z ring recomputed / re-read per chunk

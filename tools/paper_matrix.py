@@ -69,6 +69,16 @@ def main():
                     bnd = kt["boundary_ms"] / max(1, kt["boundary_launches"])
                     oth = kt["other_ms"] / max(1, kt["other_launches"])
                     step = vol + bnd + oth
+                    # the same room with temporal blocking (two steps per sweep)
+                    r.set_temporal_blocking(2)
+                    r.step(2 * (a.warmup // 2 + 1))
+                    r.synchronize()
+                    r.set_profiling(True)
+                    n2 = 2 * (a.steps // 2)
+                    r.step(n2)
+                    k2 = r.get_kernel_times()
+                    r.set_profiling(False)
+                    step2 = (k2["volume_ms"] + k2["boundary_ms"] + k2["other_ms"] + k2["shell_ms"]) / n2
                     nb, nin = info["n_boundary"], info["n_inside"]
                     key = "table_v_fimm_boundary_only" if MB == 0 else "table_vi_fdmm_mb3_boundary_only"
                     pb = paper_best(tables, key, int(size), shape, prec)
@@ -81,6 +91,7 @@ def main():
                            "volume_gvox_s": round(nin / (vol * 1e-3) / 1e9, 2),
                            "boundary_gpts_s": round(nb / (bnd * 1e-3) / 1e9, 2),
                            "step_algorithmic_gbs": round(info["bytes_per_step"] / (step * 1e-3) / 1e9, 1),
+                           "tb2_step_ms": round(step2, 4), "tb2_step_gvox_s": round(nin / (step2 * 1e-3) / 1e9, 2),
                            "paper_boundary_best": pb, "paper_fi_one_kernel_best": pv}
                     if pb:
                         row["boundary_speedup_vs_paper_best"] = round(pb["ms"] / bnd, 1)
@@ -122,20 +133,23 @@ def main():
     os.makedirs(os.path.join(ROOT, "profiles"), exist_ok=True)
     json.dump(out, open(os.path.join(ROOT, "profiles", f"{a.tag}_paper_matrix.json"), "w"), indent=1)
     lines = ["| room | shape | boundary | prec | Nb | volume ms | boundary ms (Gpts/s) | step ms (Gvox/s) | "
-             "paper best boundary ms (GPU, PAPER.md line) | paper best FI one-kernel ms |",
-             "|---|---|---|---|---|---|---|---|---|---|"]
+             "step ms, 2 steps/sweep (Gvox/s) | paper best boundary ms (GPU, PAPER.md line) | "
+             "paper best FI one-kernel ms |",
+             "|---|---|---|---|---|---|---|---|---|---|---|"]
     for r in out:
         pb = r["paper_boundary_best"]
         pv = r["paper_fi_one_kernel_best"]
         lines.append(f"| {r['room']} | {r['shape']} | {r['boundary']} | fp{r['precision']} | {r['n_boundary']} | "
                      f"{r['volume_ms']} | " + (f"{r['boundary_ms']} ({r['boundary_gpts_s']})" if r['boundary_gpts_s'] else "—") +
                      f" | {r['step_ms']} ({r['step_gvox_s']}) | "
+                     + (f"{r['tb2_step_ms']} ({r['tb2_step_gvox_s']})" if r.get('tb2_step_ms') else "—") + " | "
                      + (f"{pb['ms']} ({pb['gpu']}, {pb['line']})" if pb else "—") + " | "
                      + (f"{pv['ms']} ({pv['gpu']}, {pv['line']})" if pv else "—") + " |")
     open(os.path.join(ROOT, "profiles", f"{a.tag}_paper_matrix.md"), "w").write(
         "# The paper's experiment matrix on one B200 (context: the paper's numbers are other GPUs)\n\n"
         "Dome rows use this build's dome (DESIGN.md R12), not the paper's (its boundary counts differ).\n"
-        "Times: CUDA events around each launch, mean over the timed steps.\n\n" + "\n".join(lines) + "\n")
+        "Times: CUDA events around each launch, mean over the timed steps.  '2 steps/sweep': the same\n"
+        "room with temporal blocking (k_volume2 + boundary + shell + source per step, DESIGN.md §6).\n\n" + "\n".join(lines) + "\n")
 
 
 if __name__ == "__main__":
