@@ -21,3 +21,58 @@ def test_reference_arm_json_line(monkeypatch):
     assert out["impl"] == "reference" and out["value"] > 0
     assert out["cpu_baseline"]["kind"] == "oracle"
     assert out["e2e"]["h2d_bytes_per_step"] == 0
+
+
+class _FakeRoom:
+    """Stands in for rafd.Room in the temporal-blocking fallback logic."""
+    def __init__(self, fits):
+        self.fits, self.tb = fits, 1
+
+    def set_temporal_blocking(self, n):
+        if n == 2 and not self.fits:
+            raise rafd.RafdError(rafd.RAFD_E_NOMEM, "cudaMalloc: out of memory")
+        self.tb = n
+
+
+def test_enable_tb_single_rank():
+    import torch
+    r = _FakeRoom(True)
+    assert bench.enable_tb(r, 2, 1, torch.device("cpu")) == 2 and r.tb == 2
+    r = _FakeRoom(False)
+    assert bench.enable_tb(r, 2, 1, torch.device("cpu")) == 1 and r.tb == 1
+    r = _FakeRoom(True)
+    assert bench.enable_tb(r, 1, 1, torch.device("cpu")) == 1 and r.tb == 1
+
+
+def _tb_worker(rank, world, port, q):
+    import os
+    import torch
+    import torch.distributed as dist
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        r = _FakeRoom(fits=rank != 1)  # rank 1 runs out of memory
+        q.put((rank, bench.enable_tb(r, 2, world, torch.device("cpu")), r.tb))
+    finally:
+        dist.destroy_process_group()
+
+
+def test_enable_tb_all_ranks_agree():
+    """A NOMEM on one rank turns temporal blocking off on every rank (slabs of
+    one room must step with the same steps_per_sweep)."""
+    import socket
+    import torch.multiprocessing as mp
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    port = s.getsockname()[1]
+    s.close()
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    procs = [ctx.Process(target=_tb_worker, args=(k, 3, port, q)) for k in range(3)]
+    for p in procs:
+        p.start()
+    res = sorted(q.get(timeout=120) for _ in range(3))
+    for p in procs:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    assert res == [(0, 1, 1), (1, 1, 1), (2, 1, 1)]

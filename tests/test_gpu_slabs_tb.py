@@ -163,3 +163,55 @@ def test_tb_group_mixed_settings_rejected():
     with pytest.raises(rafd.RafdError) as e:
         rafd.rafd_step_group(slabs, 4)
     assert e.value.code == rafd.RAFD_E_STATE
+
+
+def test_tb_slabs_mode_switching_and_checkpoint(orc):
+    """Slabs switching 1 -> 2 -> 1 -> 2 steps per sweep mid-run (the state
+    moves between buffer pairs), then a checkpoint of every slab restored into
+    fresh slabs with a different z split: equal to the oracle throughout."""
+    dims = (50, 40, 23)
+    mask, mm, beta0, D, E, F = make_case("dome", dims, 2, 3, seed=7)
+    src = (25, 20, 7)
+    rcv = [(25, 20, 7), (10, 15, 15), (30, 25, 2)]
+    sig = I.gaussian_pulse(50, 4.0)
+    o = orc.OracleRoom(mask, LAM, 32, beta0, D, E, F, matmap=mm)
+    o.set_source(src, sig)
+    o.set_receivers(rcv)
+
+    def make(plan):
+        ss = [rafd.Room(mask, LAM, 32, beta0, D, E, F, matmap=mm, rank=k, nranks=len(plan), z_begin=a, z_end=b)
+              for k, (a, b) in enumerate(plan)]
+        for s in ss:
+            s.set_source(src, sig)
+            s.set_receivers(rcv)
+        return ss
+
+    plan = [(0, 6), (6, 8), (8, 16), (16, 23)]
+    slabs = make(plan)
+    for n, tb in ((7, 1), (10, 2), (3, 1), (21, 2)):
+        for s in slabs:
+            s.set_temporal_blocking(tb)
+        rafd.rafd_step_group(slabs, n)
+        o.step(n)
+        assert np.array_equal(o.read_field()[0], np.concatenate([s.read_field()[0] for s in slabs]))
+    rs = rafd.gather_receivers([s.read_receivers() for s in slabs], rcv, plan)
+    assert np.array_equal(o.read_receivers().astype(np.float32), rs.astype(np.float32))
+    # checkpoint every slab, restore into a different split (temporal blocking on)
+    cur = np.concatenate([s.read_field()[0] for s in slabs])
+    prv = np.concatenate([s.read_field()[1] for s in slabs])
+    v = np.concatenate([s.read_branch_state()[0] for s in slabs], axis=1)
+    g = np.concatenate([s.read_branch_state()[1] for s in slabs], axis=1)
+    nsteps = slabs[0].get_info()["steps"]
+    plan2 = [(0, 11), (11, 12), (12, 23)]
+    slabs2 = make(plan2)
+    off = 0
+    for s in slabs2:
+        s.set_temporal_blocking(2)
+        n = s.nb
+        s.set_state(prv, cur, v[:, off:off + n], g[:, off:off + n])
+        s.set_step(nsteps)
+        off += n
+    rafd.rafd_step_group(slabs2, 33)
+    o.step(33)
+    assert np.array_equal(o.read_field()[0], np.concatenate([s.read_field()[0] for s in slabs2]))
+    assert np.array_equal(o.read_field()[1], np.concatenate([s.read_field()[1] for s in slabs2]))
