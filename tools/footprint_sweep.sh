@@ -2,7 +2,7 @@
 # k_volume2 (tb 2) vs the single-step kernel (tb 1) over box rooms of growing footprint: tools/footprint_sweep.sh
 for d in 1536,1024,704 2048,1536,704 1536,1024,2560 2048,1536,1280 2048,1536,2560 1024,1024,2048 3072,1024,704; do
  for tb in 2 1; do
-  timeout 600 python tools/profile_run.py --config C4 --dims $d --tb $tb --steps 10 2>&1 | tail -1 | python -c "
+  timeout 600 python tools/profile_run.py --config C4 --dims $d --tb $tb --warmup 4 --steps 10 2>&1 | tail -1 | python -c "
 import sys, ast
 l = sys.stdin.read(); d = ast.literal_eval(l.split(' ', 2)[2])
 nx,ny,nz=[int(v) for v in '$d'.split(',')]

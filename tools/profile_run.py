@@ -18,6 +18,7 @@ ap.add_argument("--config", default="C4")
 ap.add_argument("--dims", default=None, help="nx,ny,nz: a box with the config's materials instead of its room")
 ap.add_argument("--steps", type=int, default=6)
 ap.add_argument("--graph", action="store_true")
+ap.add_argument("--warmup", type=int, default=0, help="untimed steps first (first launches touch fresh pages)")
 ap.add_argument("--tb", type=int, default=2, choices=[1, 2], help="steps per sweep (temporal blocking)")
 a = ap.parse_args()
 cfg = bench.workload(a.config, 1)
@@ -33,6 +34,9 @@ if a.tb == 2:
     room.set_temporal_blocking(2)
 room.set_source(I.source_position((nx, ny, nz)), I.impulse())
 room.set_receivers(I.receiver_positions((nx, ny, nz)))
+if a.warmup:
+    room.step(a.warmup)
+    room.synchronize()
 room.set_profiling(not a.graph)
 room.step(a.steps)
 room.synchronize()
