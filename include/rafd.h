@@ -160,7 +160,11 @@ int rafd_set_receivers(rafd_room *r, int32_t n, const int32_t *xyz);
 /* Initial state.  u_prev = u^{n-1}, u_curr = u^n: host or device, T-typed
  * [nz][ny][nx] of the whole room (a slab handle reads its planes); values at
  * outside voxels are ignored and stored as +0.  v, g: host or device, T-typed
- * [MB][Nb] branch state (ci = b*Nb + i).  NULL => unchanged. */
+ * [MB][Nb] branch state (ci = b*Nb + i).  NULL => unchanged.
+ * Device inputs (here and in rafd_create) may have been produced on any of the
+ * caller's streams: the call first waits for the whole device
+ * (cudaDeviceSynchronize), then copies on the room's own stream, and returns
+ * when the copies are complete -- setup calls, never on the step path. */
 int rafd_set_state(rafd_room *r, const void *u_prev, const void *u_curr, const void *v, const void *g);
 
 /* Checkpoint / resume: the state of a room is (u^n, u^{n-1}, v, g, step

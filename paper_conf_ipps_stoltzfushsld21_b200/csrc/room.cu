@@ -452,6 +452,9 @@ extern "C" int rafd_create(const rafd_room_desc *d, rafd_room **out)
     }
     if (d->device < 0 || d->device >= ndev) return set_err(RAFD_E_INVAL, "device %d out of range", d->device);
     CK(cudaSetDevice(d->device));
+    // device inputs may still be in flight on any of the caller's streams: the
+    // room's stream is non-blocking, so wait for the device first (setup call)
+    if (is_device_ptr(d->mask) || (d->matmap && is_device_ptr(d->matmap))) CK(cudaDeviceSynchronize());
     // L2 fetch granularity (experiment knob; device-wide, so opt-in only)
     if (const char *lf = getenv("RAFD_L2_FETCH")) cudaDeviceSetLimit(cudaLimitMaxL2FetchGranularity, (size_t)atoi(lf));
     rafd_room *r = new rafd_room();
@@ -1386,6 +1389,12 @@ extern "C" int rafd_set_state(rafd_room *r, const void *u_prev, const void *u_cu
     if (!r) return set_err(RAFD_E_INVAL, "null room");
     CK(cudaSetDevice(r->device));
     CK(cudaStreamSynchronize(r->stream));
+    // device inputs may still be in flight on the caller's streams (see rafd_create)
+    for (const void *p : {u_prev, u_curr, v, g})
+        if (p && is_device_ptr(p)) {
+            CK(cudaDeviceSynchronize());
+            break;
+        }
     int rc = RAFD_OK;
     const int bc = r->pair + r->cur, bp = r->pair + (r->cur ^ 1);
     if (u_prev) {

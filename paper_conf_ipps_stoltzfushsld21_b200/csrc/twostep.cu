@@ -155,11 +155,11 @@ static __device__ __forceinline__ void vol_vec(const T *c, const T *ym, const T 
 
 // The two-step kernel.  umap: u^n (box UROW x (TY+4)); pmap: u^{n-1} (TX x
 // (TY+2)); kmap: K (TX x (TY+2)); out1 = u^{n+1}, out2 = u^{n+2} (other pair).
-template <typename T, int TY, int SU, int SP>
+template <typename T, int TY, int SU, int SP, bool DYN>
 __global__ void __launch_bounds__(TbGeom<T, TY, SU, SP>::NT, 1)
     k_volume2(const __grid_constant__ CUtensorMap umap, const __grid_constant__ CUtensorMap pmap,
               const __grid_constant__ CUtensorMap kmap, T *__restrict__ out1, T *__restrict__ out2, Grid g, T l2,
-              int z_lo, int z_hi, int zchunk, int tiles_x, int tiles_y)
+              int z_lo, int z_hi, int zchunk, int tiles_x, int tiles_y, unsigned int *work)
 {
     using G = TbGeom<T, TY, SU, SP>;
     using KW = typename Vec16<T>::K;
@@ -193,7 +193,21 @@ __global__ void __launch_bounds__(TbGeom<T, TY, SU, SP>::NT, 1)
     const int units = nchunks * tiles;
     // this warp's two step-(n+1) rows, relative to the tile's first core row
     const int r0 = 2 * warp - 1;
-    for (int unit = blockIdx.x; unit < units; unit += gridDim.x) {
+    // Units in (chunk, tile-y, tile-x) order, handed out dynamically (work != null:
+    // an atomic counter, reset by the last CTA) so the units in flight stay the
+    // next ~gridDim.x ones and neighbouring tiles march their planes together; or
+    // statically round-robin.  Each CTA reserves its next unit when it starts one.
+    int *const s_next = (int *)(bar + SU + SP);
+    int unit = blockIdx.x, next_unit = 0;
+    if constexpr (DYN) {
+        if (tid == 0) *s_next = (int)atomicAdd(work, 1u);
+        __syncthreads();
+        unit = *s_next;
+    }
+    while (unit < units) {
+        if constexpr (DYN) {
+            if (tid == 0) next_unit = (int)atomicAdd(work, 1u);
+        }
         const int chunk = unit / tiles, t = unit % tiles;
         const int ty = t / tiles_x, tx = t % tiles_x;
         const int pa = 1 + z_lo + chunk * zchunk;   // first padded plane stored
@@ -323,6 +337,20 @@ __global__ void __launch_bounds__(TbGeom<T, TY, SU, SP>::NT, 1)
                 if (q + SU <= pb + 1) issue_u(q + SU);  // into the slot of plane q
                 if (q + SP <= pb) issue_pk(q + SP);
             }
+        }
+        if constexpr (DYN) {
+            if (tid == 0) *s_next = next_unit;
+            __syncthreads();
+            unit = *s_next;
+        } else {
+            unit += gridDim.x;
+        }
+    }
+    if (DYN && tid == 0) {
+        __threadfence();
+        if (atomicAdd(work + 1, 1u) == gridDim.x - 1) {  // every CTA has taken its last unit
+            atomicExch(work, 0u);
+            atomicExch(work + 1, 0u);
         }
     }
 }
@@ -463,7 +491,23 @@ struct TwoStepPlan {
     int64_t sh_lo = 0, sh_hi = 0;  // list range of the local planes [1, lnz-1) (slab interior)
     int64_t *src = nullptr;  // [7] the source's star, -1 = none
     bool idx64 = false;
+    unsigned int *work = nullptr;  // [2] dynamic unit counter, CTAs done
 };
+
+// dynamic unit scheduling in k_volume2 (RAFD_TB_DYNAMIC = 0 selects the static
+// round-robin).  Measured (same box, A/B, ms per launch): C4 3.415 -> 3.277,
+// 3072x1024x704 7.70 -> 6.47, C5 2048x1536x2560 34.9 -> 28.9: under the static
+// order a CTA that falls behind processes its tiles rounds after their
+// neighbours, whose shared halo rows have then left L2.
+static int tb_dynamic_env()
+{
+    static int v = -2;
+    if (v == -2) {
+        const char *e = getenv("RAFD_TB_DYNAMIC");
+        v = e ? (atoi(e) != 0) : 1;
+    }
+    return v;
+}
 
 template <typename T>
 cudaError_t twostep_plan_create(const Grid &g, void *const u[4], uint8_t *K_alloc, const uint8_t *K, bool idx64,
@@ -486,8 +530,11 @@ cudaError_t twostep_plan_create(const Grid &g, void *const u[4], uint8_t *K_allo
     pl->tiles_y = (g.ny + kTbTY - 1) / kTbTY;
     pl->smem = G::SMEM;
     pl->idx64 = idx64;
-    auto kern = k_volume2<T, kTbTY, kTbSU, kTbSP>;
+    auto kern = k_volume2<T, kTbTY, kTbSU, kTbSP, false>;
     cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, pl->smem);
+    if (e == cudaSuccess)
+        e = cudaFuncSetAttribute(k_volume2<T, kTbTY, kTbSU, kTbSP, true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                 pl->smem);
     int occ = 0;
     if (e == cudaSuccess) e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kern, G::NT, pl->smem);
     if (e == cudaSuccess && occ < 1) e = cudaErrorInvalidConfiguration;
@@ -520,6 +567,8 @@ cudaError_t twostep_plan_create(const Grid &g, void *const u[4], uint8_t *K_allo
         else k_shell_compact<uint32_t><<<blocks, 256, 0, s>>>(g, K, off, (uint32_t *)pl->list);
         e = cudaGetLastError();
     }
+    if (e == cudaSuccess) e = cudaMalloc(&pl->work, 2 * sizeof(unsigned int));
+    if (e == cudaSuccess) e = cudaMemsetAsync(pl->work, 0, 2 * sizeof(unsigned int), s);
     if (e == cudaSuccess) e = cudaMalloc(&pl->src, 7 * 8);
     if (e == cudaSuccess) e = cudaMemsetAsync(pl->src, 0xff, 7 * 8, s);
     if (e == cudaSuccess) e = cudaStreamSynchronize(s);
@@ -530,6 +579,7 @@ cudaError_t twostep_plan_create(const Grid &g, void *const u[4], uint8_t *K_allo
     if (e != cudaSuccess) {
         if (pl->list) cudaFree(pl->list);
         if (pl->src) cudaFree(pl->src);
+        if (pl->work) cudaFree(pl->work);
         delete pl;
         return e;
     }
@@ -544,6 +594,7 @@ void twostep_plan_destroy(void *plan)
     if (!pl) return;
     if (pl->list) cudaFree(pl->list);
     if (pl->src) cudaFree(pl->src);
+    if (pl->work) cudaFree(pl->work);
     delete pl;
 }
 
@@ -604,9 +655,15 @@ cudaError_t launch_volume2(const void *plan, const Grid &g, int cur_buf, int pre
     const int zc = tb_choose_zchunk(z_hi - z_lo, tiles, pl->grid);
     const long units = (long)tiles * ((z_hi - z_lo + zc - 1) / zc);
     const int grid = (int)std::min<long>(pl->grid, units);
-    k_volume2<T, kTbTY, kTbSU, kTbSP><<<grid, G::NT, pl->smem, s>>>(pl->umap[cur_buf], pl->pmap[prev_buf], pl->kmap,
-                                                                    out1, out2, g, l2, z_lo, z_hi, zc, pl->tiles_x,
-                                                                    pl->tiles_y);
+    const int env = tb_dynamic_env();
+    if (env)
+        k_volume2<T, kTbTY, kTbSU, kTbSP, true><<<grid, G::NT, pl->smem, s>>>(
+            pl->umap[cur_buf], pl->pmap[prev_buf], pl->kmap, out1, out2, g, l2, z_lo, z_hi, zc, pl->tiles_x,
+            pl->tiles_y, pl->work);
+    else
+        k_volume2<T, kTbTY, kTbSU, kTbSP, false><<<grid, G::NT, pl->smem, s>>>(
+            pl->umap[cur_buf], pl->pmap[prev_buf], pl->kmap, out1, out2, g, l2, z_lo, z_hi, zc, pl->tiles_x,
+            pl->tiles_y, nullptr);
     return cudaGetLastError();
 }
 
