@@ -610,14 +610,16 @@ cudaError_t twostep_set_source(void *plan, int64_t pos, const Grid &g)
     return cudaMemcpy(pl->src, h, sizeof h, cudaMemcpyHostToDevice);
 }
 
-// Cap on the planes one unit marches (RAFD_TB_ZCHUNK_MAX, default 0 = none):
-// long marches let the CTAs drift apart in z.
+// Cap on the planes one unit marches (RAFD_TB_ZCHUNK_MAX, 0 = none; default
+// 256).  Measured with dynamic scheduling, ms per launch: C5 (chunk 366
+// uncapped) 28.4 -> 24.3 at 256; C4 (118) and 3072x1024x704 (235) unchanged;
+// 64-176 cost C4 / 3072x1024x704 1-2 % (the z ring restarts per unit).
 static int tb_zchunk_cap()
 {
     static int v = -1;
     if (v < 0) {
         const char *e = getenv("RAFD_TB_ZCHUNK_MAX");
-        v = e ? std::max(0, atoi(e)) : 0;
+        v = e ? std::max(0, atoi(e)) : 256;
     }
     return v;
 }
