@@ -84,6 +84,9 @@ template <typename T> struct FusedArgs {
     // halo push: byte offsets from an output address to the
     // same voxel in a neighbour's ghost plane (peer memory); 0 = no mirror
     int64_t mirror[2];
+    // dynamic unit scheduling (set by the plan): [2] atomic unit counter and
+    // CTAs-done count, reset by the last CTA; nullptr = static round-robin
+    unsigned int *work;
 };
 
 // plan == nullptr selects the one-thread-per-voxel v0 kernel (A/B reference);
