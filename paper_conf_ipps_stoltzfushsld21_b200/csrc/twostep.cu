@@ -494,8 +494,8 @@ struct TwoStepPlan {
     unsigned int *work = nullptr;  // [2] dynamic unit counter, CTAs done
 };
 
-// dynamic unit scheduling in k_volume2 (RAFD_TB_DYNAMIC = 0 selects the static
-// round-robin).  Measured (same box, A/B, ms per launch): C4 3.415 -> 3.277,
+// dynamic unit scheduling in k_volume2 (RAFD_TB_DYNAMIC = 0 never, 1 always,
+// unset: units of >= 24 planes).  Measured (same box, A/B, ms per launch): C4 3.415 -> 3.277,
 // 3072x1024x704 7.70 -> 6.47, C5 2048x1536x2560 34.9 -> 28.9: under the static
 // order a CTA that falls behind processes its tiles rounds after their
 // neighbours, whose shared halo rows have then left L2.
@@ -504,10 +504,11 @@ static int tb_dynamic_env()
     static int v = -2;
     if (v == -2) {
         const char *e = getenv("RAFD_TB_DYNAMIC");
-        v = e ? (atoi(e) != 0) : 1;
+        v = e ? (atoi(e) != 0) : -1;
     }
     return v;
 }
+static constexpr int kTbDynMinChunk = 24;  // unset: dynamic for units of >= 24 planes (small rooms stay static)
 
 template <typename T>
 cudaError_t twostep_plan_create(const Grid &g, void *const u[4], uint8_t *K_alloc, const uint8_t *K, bool idx64,
@@ -658,7 +659,7 @@ cudaError_t launch_volume2(const void *plan, const Grid &g, int cur_buf, int pre
     const long units = (long)tiles * ((z_hi - z_lo + zc - 1) / zc);
     const int grid = (int)std::min<long>(pl->grid, units);
     const int env = tb_dynamic_env();
-    if (env)
+    if (env == 1 || (env < 0 && zc >= kTbDynMinChunk))
         k_volume2<T, kTbTY, kTbSU, kTbSP, true><<<grid, G::NT, pl->smem, s>>>(
             pl->umap[cur_buf], pl->pmap[prev_buf], pl->kmap, out1, out2, g, l2, z_lo, z_hi, zc, pl->tiles_x,
             pl->tiles_y, pl->work);

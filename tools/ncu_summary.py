@@ -1,7 +1,7 @@
 """Summarise ncu captures for profiles/ (run here, no GPU needed).
 
     python tools/ncu_summary.py launches <launches.csv>      # per-kernel share of the step
-    python tools/ncu_summary.py full <report.ncu-rep>        # key metrics of one capture
+    python tools/ncu_summary.py full <report.ncu-rep> [name]  # key metrics of one capture
 """
 import csv
 import io
@@ -51,11 +51,16 @@ def launches(path):
     return out
 
 
-def full(path):
+def full(path, match=None):
+    """Key metrics of the first capture whose kernel name contains `match`."""
     raw = subprocess.run(["ncu", "-i", path, "--page", "raw", "--csv"], capture_output=True, text=True).stdout
     r = list(csv.reader(io.StringIO(raw)))
-    h, units, v = r[0], r[1], r[2]
-    out = {"kernel": v[h.index("Kernel Name")] if "Kernel Name" in h else None}
+    h, units = r[0], r[1]
+    rows = r[2:]
+    if match:
+        rows = [v for v in rows if match in v[h.index("Kernel Name")]]
+    v = rows[0]
+    out = {"kernel": v[h.index("Kernel Name")] if "Kernel Name" in h else None, "source": path.split("/")[-1]}
     for k in KEYS:
         if k in h:
             i = h.index(k)
@@ -65,4 +70,5 @@ def full(path):
 
 if __name__ == "__main__":
     mode, path = sys.argv[1], sys.argv[2]
-    print(json.dumps(launches(path) if mode == "launches" else full(path), indent=1))
+    match = sys.argv[3] if len(sys.argv) > 3 else None
+    print(json.dumps(launches(path) if mode == "launches" else full(path, match), indent=1))
