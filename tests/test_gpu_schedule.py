@@ -1,6 +1,7 @@
 """Unit scheduling of the two volume kernels: dynamic (atomic
 unit counter, self-resetting) or static round-robin must give the same bits.
-Small rooms default to static and large ones to dynamic, so each test forces
+Small rooms default to static and large ones to dynamic (and skip the K plane
+of uniform tile-planes only when large), so each test forces
 one mode in a fresh process (the choice is read once per process) and checks
 the single-step and two-step paths against the oracle, over several launches
 (the counter must reset between them) and a slab group."""
@@ -56,7 +57,9 @@ print("ok")
 
 @pytest.mark.parametrize("mode", ["0", "1"])
 def test_dynamic_and_static_scheduling_bitwise(mode):
-    env = dict(os.environ, RAFD_VOL_DYNAMIC=mode, RAFD_TB_DYNAMIC=mode, RAFD_FUSED="0")
+    # RAFD_K6: the K-plane skip of uniform tile-planes (default only in rooms of
+    # >= 2^28 voxels) is exercised on this small room too
+    env = dict(os.environ, RAFD_VOL_DYNAMIC=mode, RAFD_TB_DYNAMIC=mode, RAFD_K6=mode, RAFD_FUSED="0")
     # short z-chunks so that the dynamic counter hands out many units per launch
     env["RAFD_ZCHUNK_MAX"] = "8"
     env["RAFD_TB_ZCHUNK_MAX"] = "8"
