@@ -255,3 +255,31 @@ def test_errors():
     with pytest.raises(rafd.RafdError):  # the halo push needs an IPC-connected slab
         g.set_halo_push(True)
     g.set_halo_push(False)
+
+
+@pytest.mark.parametrize("precision,MB,shape,dims", [(32, 0, "lshape", (96, 88, 80)), (32, 3, "dome", (90, 84, 76)),
+                                                   (64, 3, "box", (70, 64, 60))])
+def test_long_run_1000_steps(orc, precision, MB, shape, dims):
+    """The north_star tolerance is stated after 1000 steps: an impulse response
+    of 1000 steps (graph replays of 16 steps plus direct double steps) with
+    temporal blocking, FI-MM on an L-shape and FD-MM on a dome / box, against
+    the oracle's single steps -- bitwise."""
+    mask_t = I.make_mask(shape, *dims)
+    M = 4 if MB == 0 else 8
+    mm = I.material_map(mask_t, "region", M).numpy()
+    mask = mask_t.numpy()
+    if MB:
+        beta0, D, E, F = I.fd_tables(M, MB)
+    else:
+        beta0, D, E, F = I.fi_beta_from_alpha([0.05, 0.2, 0.5, 0.9]), None, None, None
+    src = I.source_position(dims, mask)
+    rcv = I.receiver_positions(dims, mask)
+    o = orc.OracleRoom(mask, LAM, precision, beta0, D, E, F, matmap=mm)
+    g = tb_room(mask, precision, beta0, D, E, F, matmap=mm)
+    for r in (o, g):
+        r.set_source(src, I.impulse())
+        r.set_receivers(rcv)
+    o.step(1000)
+    g.step(998)
+    g.step(2)
+    compare(o, g, precision, branches=bool(MB))
