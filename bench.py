@@ -313,6 +313,9 @@ def run_rafd(args, rank, world, local_rank):
                 "l2": "inputs larger than L2 (working set %.1f GB/GPU vs 126 MB L2)" % (info["device_bytes"] / 1e9),
                 "timed": "profiled launches (CUDA events around every kernel) on the room stream",
                 "steps_per_sweep": tb,
+                # RAFD_BENCH_DEVICE pins every rank to one GPU (a functional check of the
+                # multi-rank path): the ranks then share that GPU's bandwidth
+                "ranks_per_gpu": world if os.environ.get("RAFD_BENCH_DEVICE") is not None else 1,
             },
             "roofline": {
                 "bound": "hbm",
