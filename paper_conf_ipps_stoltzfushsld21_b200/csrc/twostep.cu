@@ -441,17 +441,23 @@ __global__ void __launch_bounds__(256) k_shell(const IdxT *__restrict__ list, in
     const int64_t p = i < n ? (int64_t)list[i] : src[i - n];
     if (p < 0) return;
     if (i >= n && (p < (int64_t)zp_lo * g.plane || p >= (int64_t)zp_hi * g.plane)) return;
+    // every load depends only on p: all of them in flight together (one
+    // dependent round trip after the list entry instead of two)
     const int nbr = K[p];
-    if (nbr == 0) return;
-    T s = R::add(u1[p - 1], u1[p + 1]);
-    s = R::add(s, u1[p - g.pitch]);
-    s = R::add(s, u1[p + g.pitch]);
-    s = R::add(s, u1[p - g.plane]);
-    s = R::add(s, u1[p + g.plane]);
+    const T xm = u1[p - 1], xp = u1[p + 1], ym = u1[p - g.pitch], yp = u1[p + g.pitch];
+    const T zm = u1[p - g.plane], zp = u1[p + g.plane], c = u1[p], pv = u0[p];
+    T s = R::add(xm, xp);
+    s = R::add(s, ym);
+    s = R::add(s, yp);
+    s = R::add(s, zm);
+    s = R::add(s, zp);
     const T a = R::sub((T)2, R::mul(l2, (T)nbr));
-    T t = R::mul(a, u1[p]);
+    T t = R::mul(a, c);
     t = R::add(t, R::mul(l2, s));
-    out[p] = R::sub(t, u0[p]);
+    // an outside voxel (a star entry with K = 0) holds +0 in every buffer, so
+    // storing u0 there changes nothing -- and the store then needs every load
+    // (the compiler cannot sink any of them below a K test)
+    out[p] = nbr != 0 ? R::sub(t, pv) : pv;
 }
 
 // ------------------------------------------------------------------ host side
