@@ -18,6 +18,7 @@ ap.add_argument("--config", default="C4")
 ap.add_argument("--dims", default=None, help="nx,ny,nz: a box with the config's materials instead of its room")
 ap.add_argument("--steps", type=int, default=6)
 ap.add_argument("--graph", action="store_true")
+ap.add_argument("--precision", type=int, default=None, choices=[32, 64])
 ap.add_argument("--warmup", type=int, default=0, help="untimed steps first (first launches touch fresh pages)")
 ap.add_argument("--tb", type=int, default=2, choices=[1, 2], help="steps per sweep (temporal blocking)")
 a = ap.parse_args()
@@ -25,6 +26,8 @@ cfg = bench.workload(a.config, 1)
 if a.dims:
     cfg["room"] = tuple(int(v) for v in a.dims.split(","))
 nx, ny, nz = cfg["room"]
+if a.precision:
+    cfg["precision"] = a.precision
 beta0, D, E, F = I.config_materials(cfg)
 mask, mm, mz0 = bench.slab_inputs(cfg, 0, nz, torch.device("cuda", 0))
 room = rafd.Room(mask, 1 / math.sqrt(3), cfg["precision"], beta0, D, E, F, matmap=mm)
