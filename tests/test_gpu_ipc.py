@@ -78,9 +78,8 @@ def _worker(rank, world, port, plan, q, push=False, tb=1):
         dist.destroy_process_group()
 
 
-@pytest.mark.parametrize("tb", [1, 2])
-@pytest.mark.parametrize("push", [False, True])
-@pytest.mark.parametrize("world", [2, 3])
+@pytest.mark.parametrize("world,push,tb", [(w, p, t) for w in (2, 3) for p in (False, True) for t in (1, 2)]
+                         + [(5, False, 2), (5, True, 2)])
 def test_ipc_slabs_equal_single_room(world, push, tb):
     """tb = 2: temporal blocking in every slab (edge planes single-step, the
     two-step kernel over the interior; two exchanges per double step)."""
