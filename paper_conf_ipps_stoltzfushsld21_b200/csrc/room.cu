@@ -111,6 +111,7 @@ struct rafd_room {
     void *tab = nullptr;   // T: beta[M] | BI | D | DI | F  ([M*MB] each)
     double *DF = nullptr;  // double D | F for the energy hook
     void *ctl = nullptr;   // Ctl<T>
+    unsigned int *ticket = nullptr;  // last-block ticket of the boundary kernel's fused source/receivers
     void *sig = nullptr;
     int64_t *rcv_pos = nullptr;
     void *rec = nullptr;
@@ -416,6 +417,8 @@ template <typename T> static int create_t(rafd_room *r, const rafd_room_desc *d)
     CK(cudaMemcpy(r->tab, tab.data(), tab.size() * sizeof(T), cudaMemcpyHostToDevice));
     CK(cudaMemcpy(r->DF, DF.data(), DF.size() * sizeof(double), cudaMemcpyHostToDevice));
     if ((rc = dmalloc(r, &r->ctl, sizeof(Ctl<T>)))) return rc;
+    if ((rc = dmalloc(r, (void **)&r->ticket, sizeof(unsigned int)))) return rc;
+    CK(cudaMemset(r->ticket, 0, sizeof(unsigned int)));
     Ctl<T> c{};
     c.src_pos = -1;
     c.src_node = -1;
@@ -534,7 +537,7 @@ extern "C" void rafd_destroy(rafd_room *r)
     if (r->vplan) volume_plan_destroy(r->vplan);
     if (r->tbplan) twostep_plan_destroy(r->tbplan);
     void *ps[] = {r->u[0], r->u[1], r->u[2], r->u[3], r->K_alloc, r->bpos, r->bidx, r->Kb, r->matb, r->ub, r->gst, r->vst,
-                  r->tab, r->DF, r->ctl, r->sig, r->rcv_pos, r->rec};
+                  r->tab, r->DF, r->ctl, r->ticket, r->sig, r->rcv_pos, r->rec};
     for (void *p : ps)
         if (p) cudaFree(p);
     for (auto &e : r->evs) {
@@ -733,16 +736,14 @@ template <typename T> static cudaError_t enqueue_step(rafd_room *r, int pair, in
     });
     if (e != cudaSuccess) return e;
     if (r->nb > 0 && !r->fused && !r->scheme) {
-        e = timed(1, [&] {
+        // the source and receivers run in the boundary kernel's last block
+        return timed(1, [&] {
             return launch_boundary<T>(r->MB, r->idx64, r->bpos, r->Kb, r->matb, 0, r->nb, r->nb, un,
                                       ub_slot<T>(r, cur), (T *)r->gst, (T *)r->vst, (const T *)r->tab, r->M,
-                                      r->lambda, s);
+                                      r->lambda, s, 0, 0, ctl_of<T>(r), r->ticket);
         });
-        if (e != cudaSuccess) return e;
     }
-    e = timed(2, [&] { return launch_src_rcv<T>(un, ub_slot<T>(r, cur), ctl_of<T>(r), s); });
-    if (e != cudaSuccess) return e;
-    return cudaSuccess;
+    return timed(2, [&] { return launch_src_rcv<T>(un, ub_slot<T>(r, cur), ctl_of<T>(r), s); });
 }
 
 // one double step of the two-step kernel (twostep.cu) from the state (pair,
@@ -754,21 +755,22 @@ template <typename T> static cudaError_t enqueue_step2(rafd_room *r, int pair, i
     const Grid &g = r->g;
     const int bA = pair + (cur ^ 1), bB = pair + cur, bC = (pair ^ 2) + (cur ^ 1), bD = (pair ^ 2) + cur;
     T *B = (T *)r->u[bB], *C = (T *)r->u[bC], *D = (T *)r->u[bD];
-    auto bnd = [&](T *un, int slot) -> cudaError_t {
-        if (r->nb == 0) return cudaSuccess;
+    // boundary update + (in its last block) source and receivers of one step;
+    // without boundary nodes the source/receiver kernel alone
+    auto bnd_src = [&](T *un, int slot) -> cudaError_t {
+        if (r->nb == 0)
+            return timed_launch(r, s, prof, 2, [&] { return launch_src_rcv<T>(un, ub_slot<T>(r, slot), ctl_of<T>(r), s); });
         return timed_launch(r, s, prof, 1, [&] {
             return launch_boundary<T>(r->MB, r->idx64, r->bpos, r->Kb, r->matb, 0, r->nb, r->nb, un,
                                       ub_slot<T>(r, slot), (T *)r->gst, (T *)r->vst, (const T *)r->tab, r->M,
-                                      r->lambda, s);
+                                      r->lambda, s, 0, 0, ctl_of<T>(r), r->ticket);
         });
     };
     cudaError_t e = timed_launch(r, s, prof, 0, [&] { return launch_volume2<T>(r->tbplan, g, bB, bA, C, D, r->lambda, s); });
-    if (e == cudaSuccess) e = bnd(C, cur);
-    if (e == cudaSuccess) e = timed_launch(r, s, prof, 2, [&] { return launch_src_rcv<T>(C, ub_slot<T>(r, cur), ctl_of<T>(r), s); });
+    if (e == cudaSuccess) e = bnd_src(C, cur);
     if (e == cudaSuccess)
         e = timed_launch(r, s, prof, 3, [&] { return launch_shell<T>(r->tbplan, g, C, B, r->K, D, r->lambda, s); });
-    if (e == cudaSuccess) e = bnd(D, cur ^ 1);
-    if (e == cudaSuccess) e = timed_launch(r, s, prof, 2, [&] { return launch_src_rcv<T>(D, ub_slot<T>(r, cur ^ 1), ctl_of<T>(r), s); });
+    if (e == cudaSuccess) e = bnd_src(D, cur ^ 1);
     return e;
 }
 
@@ -987,8 +989,10 @@ static cudaError_t slab_step(rafd_room *r, bool two, bool prof, int64_t n)
     return e;
 }
 
-static int kernels_per_step(const rafd_room *r) { return 2 + (r->nb > 0 && !r->fused && !r->scheme ? 1 : 0); }
-static int kernels_per_double_step(const rafd_room *r) { return 4 + (r->nb > 0 ? 2 : 0); }
+// (whole room: the boundary kernel runs the source/receivers in its last block;
+// fused / single-kernel schemes and rooms without boundary nodes launch k_src_rcv)
+static int kernels_per_step(const rafd_room *) { return 2; }
+static int kernels_per_double_step(const rafd_room *) { return 4; }
 
 // a graph of G steps from the state (pair, cur) (index pair + cur); it ends in
 // the same state (G single steps flip cur an even number of times, G/2 double

@@ -241,7 +241,7 @@ def test_graph_direct_and_single_step_agree(orc):
     assert t["volume_launches"] == 34 and t["shell_launches"] == 33 and t["boundary_launches"] == 67
     assert np.array_equal(a.read_field()[0], b.read_field()[0])
     assert np.array_equal(a.read_field()[0], c.read_field()[0])
-    assert a.launch_count() == b.launch_count() == 33 * 6 + 3
+    assert a.launch_count() == b.launch_count() == 33 * 4 + 2  # k_volume2, 2 boundary (+src/rcv), shell
 
 
 def test_errors():
