@@ -149,7 +149,9 @@ def main():
         "# The paper's experiment matrix on one B200 (context: the paper's numbers are other GPUs)\n\n"
         "Dome rows use this build's dome (DESIGN.md R12), not the paper's (its boundary counts differ).\n"
         "Times: CUDA events around each launch, mean over the timed steps.  '2 steps/sweep': the same\n"
-        "room with temporal blocking (k_volume2 + boundary + shell + source per step, DESIGN.md §6).\n\n" + "\n".join(lines) + "\n")
+        "room with temporal blocking (k_volume2 + boundary + shell + source per step, DESIGN.md §6).\n"
+        "The boundary kernel also injects the source and records the receivers in its last block\n"
+        "(whole-room steps, DESIGN.md §6): its column includes that tail (~2 us).\n\n" + "\n".join(lines) + "\n")
 
 
 if __name__ == "__main__":
