@@ -801,16 +801,20 @@ static cudaError_t enqueue_phase(rafd_room *r, int phase, cudaStream_t s, bool p
                                     (r->fused || r->scheme || m0 || m1) ? &f : nullptr);
         });
     };
-    auto bnd = [&](int64_t lo, int64_t hi, int64_t m0, int64_t m1) -> cudaError_t {
+    auto bnd = [&](int64_t lo, int64_t hi, int64_t m0, int64_t m1, int src_mode = 0) -> cudaError_t {
         if (hi <= lo || r->fused || r->scheme) return cudaSuccess;
         return timed(1, [&] {
             return launch_boundary<T>(r->MB, r->idx64, r->bpos, r->Kb, r->matb, lo, hi, r->nb, un,
                                       ub_slot<T>(r, cur), (T *)r->gst, (T *)r->vst, (const T *)r->tab, r->M,
-                                      r->lambda, s, m0, m1);
+                                      r->lambda, s, m0, m1, src_mode ? ctl_of<T>(r) : nullptr, r->ticket,
+                                      src_mode);
         });
     };
     const int zs = r->src_z >= 0 ? r->src_z - r->z0 : -1;
     const bool src_edge = zs == 0 || zs == lnz - 1;
+    // the interior phase's source/receivers run in the interior boundary kernel's
+    // last block when that kernel runs
+    const bool bnd_src = !r->fused && !r->scheme && lnz > 2 && r->n_last_start > r->n_first_plane;
     cudaError_t e = cudaSuccess;
     if (phase == 0) {
         e = vol(0, 1, mf0, mf1);
@@ -822,8 +826,9 @@ static cudaError_t enqueue_phase(rafd_room *r, int phase, cudaStream_t s, bool p
             e = timed(2, [&] { return launch_src_rcv<T>(un, ub_slot<T>(r, cur), ctl_of<T>(r), s, 1, ms0, ms1); });
     } else {
         if (lnz > 2) e = vol(1, lnz - 1, 0, 0);
-        if (e == cudaSuccess && lnz > 2) e = bnd(r->n_first_plane, r->n_last_start, 0, 0);
-        if (e == cudaSuccess) e = timed(2, [&] { return launch_src_rcv<T>(un, ub_slot<T>(r, cur), ctl_of<T>(r), s, src_edge ? 2 : 3); });
+        if (e == cudaSuccess && lnz > 2) e = bnd(r->n_first_plane, r->n_last_start, 0, 0, bnd_src ? (src_edge ? 2 : 3) : 0);
+        if (e == cudaSuccess && !bnd_src)
+            e = timed(2, [&] { return launch_src_rcv<T>(un, ub_slot<T>(r, cur), ctl_of<T>(r), s, src_edge ? 2 : 3); });
     }
     return e;
 }
@@ -838,7 +843,9 @@ static int kernels_per_phase(const rafd_room *r, int phase)
                nbk * (lnz > 1 && r->nb > std::max(r->n_last_start, r->n_first_plane) ? 1 : 0) +
                ((zs == 0 || zs == lnz - 1) ? 1 : 0);
     }
-    return (lnz > 2 ? 1 : 0) + nbk * (lnz > 2 && r->n_last_start > r->n_first_plane ? 1 : 0) + 1;
+    // interior volume, then either the interior boundary kernel (which runs the
+    // source/receivers in its last block) or k_src_rcv alone
+    return (lnz > 2 ? 1 : 0) + 1;
 }
 
 // ---- slab double step under temporal blocking (twostep.cu), from the state
@@ -882,13 +889,15 @@ static cudaError_t enqueue_tb_phase(rafd_room *r, int ph, cudaStream_t s, bool p
                                     (m0 || m1) ? &f : nullptr, bp);
         });
     };
-    auto bnd = [&](int64_t lo, int64_t hi, int64_t m0, int64_t m1) -> cudaError_t {
+    auto bnd = [&](int64_t lo, int64_t hi, int64_t m0, int64_t m1, int src_mode = 0) -> cudaError_t {
         if (hi <= lo) return cudaSuccess;
         return timed(1, [&] {
             return launch_boundary<T>(r->MB, r->idx64, r->bpos, r->Kb, r->matb, lo, hi, r->nb, out, ub, (T *)r->gst,
-                                      (T *)r->vst, (const T *)r->tab, r->M, r->lambda, s, m0, m1);
+                                      (T *)r->vst, (const T *)r->tab, r->M, r->lambda, s, m0, m1,
+                                      src_mode ? ctl_of<T>(r) : nullptr, r->ticket, src_mode);
         });
     };
+    const bool bnd_src = lnz > 2 && r->n_last_start > r->n_first_plane;  // see enqueue_phase
     const int zs = r->src_z >= 0 ? r->src_z - r->z0 : -1;
     const bool src_edge = zs == 0 || zs == lnz - 1;
     cudaError_t e = cudaSuccess;
@@ -913,8 +922,9 @@ static cudaError_t enqueue_tb_phase(rafd_room *r, int ph, cudaStream_t s, bool p
                                            (T *)r->u[bD], r->lambda, s, true);
                 });
         }
-        if (e == cudaSuccess && lnz > 2) e = bnd(r->n_first_plane, r->n_last_start, 0, 0);
-        if (e == cudaSuccess)
+        if (e == cudaSuccess && lnz > 2)
+            e = bnd(r->n_first_plane, r->n_last_start, 0, 0, bnd_src ? (src_edge ? 2 : 3) : 0);
+        if (e == cudaSuccess && !bnd_src)
             e = timed(2, [&] { return launch_src_rcv<T>(out, ub, ctl_of<T>(r), s, src_edge ? 2 : 3); });
     }
     return e;
