@@ -362,6 +362,13 @@ def enable_tb(room, want, world, dev):
     fits (C5 fp32 on one GPU needs ~143 GB); every rank must run the same
     setting, so a NOMEM anywhere falls back to single steps everywhere."""
     from paper_conf_ipps_stoltzfushsld21_b200 import rafd
+    if want == 0:
+        info = room.get_info()
+        want = 2 if info["n_mask"] >= (1 << 25) else 1
+        if world > 1:  # every rank decides alike (slabs of one room share the setting)
+            t = torch.tensor([want], dtype=torch.int32, device=dev)
+            torch.distributed.all_reduce(t, op=torch.distributed.ReduceOp.MIN)
+            want = int(t[0])
     tb = 1
     if want == 2:
         try:
@@ -513,8 +520,10 @@ def main():
     ap.add_argument("--config", default="C4")
     ap.add_argument("--precision", type=int, default=None)
     ap.add_argument("--no-cpu-baseline", action="store_true")
-    ap.add_argument("--tb", type=int, default=2, choices=[1, 2],
-                    help="steps per HBM sweep (temporal blocking; whole rooms on one GPU only)")
+    ap.add_argument("--tb", type=int, default=0, choices=[0, 1, 2],
+                    help="steps per HBM sweep (2: temporal blocking); 0 = auto: 2 for rooms of >= 2^25 "
+                         "voxels per GPU, 1 below (measured: C2 256^3 is faster with single steps, C3 and "
+                         "up with two, profiles/r01_other_configs.txt)")
     ap.add_argument("--transport", default="nccl", choices=["nccl", "ipc", "push"],
                     help="halo exchange for --gpus > 1: NCCL send/recv, or CUDA-IPC peer copies "
                          "ordered by GPU-side stream waits (rafd_ipc_connect)")

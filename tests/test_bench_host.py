@@ -25,8 +25,11 @@ def test_reference_arm_json_line(monkeypatch):
 
 class _FakeRoom:
     """Stands in for rafd.Room in the temporal-blocking fallback logic."""
-    def __init__(self, fits):
-        self.fits, self.tb = fits, 1
+    def __init__(self, fits, n_mask=1 << 30):
+        self.fits, self.tb, self.n_mask = fits, 1, n_mask
+
+    def get_info(self):
+        return {"n_mask": self.n_mask}
 
     def set_temporal_blocking(self, n):
         if n == 2 and not self.fits:
@@ -42,6 +45,9 @@ def test_enable_tb_single_rank():
     assert bench.enable_tb(r, 2, 1, torch.device("cpu")) == 1 and r.tb == 1
     r = _FakeRoom(True)
     assert bench.enable_tb(r, 1, 1, torch.device("cpu")) == 1 and r.tb == 1
+    # auto: two steps per sweep from 2^25 voxels on (C3 and up), single steps below (C2)
+    assert bench.enable_tb(_FakeRoom(True, 1536 * 1024 * 704), 0, 1, torch.device("cpu")) == 2
+    assert bench.enable_tb(_FakeRoom(True, 256 ** 3), 0, 1, torch.device("cpu")) == 1
 
 
 def _tb_worker(rank, world, port, q):
