@@ -276,6 +276,77 @@ def test_energy_decays_lossy(orc, room):
     assert h[-1] < 0.99 * h[0]
 
 
+def _balance_rhs(mask, K, bidx, lam, beta0, D, E, F, matb, u_prev, u_next, v0, v1, g0, g1):
+    """Right-hand side of the exact one-step energy balance (SURVEY.md Appendix
+    A.1, reading R11), from the fields and branch states alone:
+      H^{n+1/2} - H^{n-1/2} = - sum_{boundary i} lam (6-K_i) [ beta0 du^2 / 2
+                              + sum_b ( 2 E_b mu_v_b^2 + F_b (g'_b - g_b)^2 ) ]
+    with du = u^{n+1} - u^{n-1} at the node and mu_v_b = (v'_b + v_b) / 2.
+    It follows from multiplying the FVTD update by du and the
+    branch ODE 2D(v'-v) + E(v'+v) + 2F g' = du (Listing 4 with R5's BI, DI;
+    PAPER.md:426-440) by mu_v."""
+    flat_prev, flat_next = u_prev.reshape(-1), u_next.reshape(-1)
+    a = lam * (6.0 - K.reshape(-1)[bidx].astype(np.float64))
+    du = flat_next[bidx].astype(np.float64) - flat_prev[bidx].astype(np.float64)
+    diss = np.asarray(beta0, np.float64)[matb] * du * du / 2.0
+    for b in range(v0.shape[0]):
+        mu = (v1[b].astype(np.float64) + v0[b].astype(np.float64)) / 2.0
+        dg = g1[b].astype(np.float64) - g0[b].astype(np.float64)
+        diss = diss + 2.0 * E[matb, b] * mu * mu + F[matb, b] * dg * dg
+    return -(a * diss).sum()
+
+
+@pytest.mark.parametrize("room", list(ROOMS))
+def test_energy_balance_exact(orc, room):
+    """Exact per-step energy balance (not just its sign): every term of the
+    oracle's H -- kinetic, edge, and the boundary D v^2 and F g^2 terms -- is
+    pinned by the dissipation computed independently from the states.  FD
+    tables with D, E, F > 0 and beta0 > 0, random field and branch state; an
+    FI room with beta0 > 0; an R-free (E = 0) table so that the F terms carry
+    the whole dissipation of the branches."""
+    mask = ROOMS[room]()
+    mm = I.material_map(I.torch.from_numpy(mask), "random", 4).numpy()
+    rng = np.random.default_rng(2024)
+    beta0, D, E, F = I.fd_tables(4, 3)
+    beta0 = np.array([0.0, 0.05, 0.3, 0.02])
+    E_free = E.copy()
+    E_free[:, :] = 0.0
+    cases = [("fi", beta0 + 0.01, None, None, None),
+             ("fd", beta0, D, E, F),
+             ("fd_E0", beta0 * 0, D, E_free, F)]
+    for name, b0, Dc, Ec, Fc in cases:
+        r = orc.OracleRoom(mask, LAM, 64, b0, Dc, Ec, Fc, matmap=mm)
+        K, bidx_c, Kb, matb = r.classification()
+        nz, ny, nx = mask.shape
+        z, rem = np.divmod(bidx_c, ny * nx)
+        y, x = np.divmod(rem, nx)
+        bflat = (z * ny + y) * nx + x
+        up, uc = _rand_state(mask, 31, np.float64)
+        nb, MB = r.nb, (0 if Dc is None else Dc.shape[1])
+        v = rng.uniform(-1, 1, (MB, nb))
+        g = rng.uniform(-1, 1, (MB, nb))
+        r.set_state(up, uc, v if MB else None, g if MB else None)
+        for _ in range(5):
+            h0 = r.energy()
+            u_n, u_prev = r.read_field()
+            v0, g0 = r.read_branch_state() if MB else (np.zeros((0, nb)), np.zeros((0, nb)))
+            r.step(1)
+            h1 = r.energy()
+            u_next, _ = r.read_field()
+            v1, g1 = r.read_branch_state() if MB else (np.zeros((0, nb)), np.zeros((0, nb)))
+            rhs = _balance_rhs(mask, K, bflat, LAM, b0, Dc if MB else None,
+                               Ec if MB else None, Fc if MB else None, matb,
+                               u_prev, u_next, v0, v1, g0, g1)
+            assert rhs < 0, name
+            assert abs((h1 - h0) - rhs) <= 1e-12 * abs(h0), (name, h1 - h0, rhs)
+            if MB:
+                # the F g^2 part of H alone is O(1) here: a dropped or scaled
+                # term would break the balance by that much
+                a = LAM * (6.0 - Kb.astype(np.float64))
+                fg = (a * (Fc[matb, :].T * g1 * g1).sum(0)).sum()
+                assert fg > 1e-3 * abs(h1), name
+
+
 # ---------------------------------------------------------------- P5 stability limit
 
 
