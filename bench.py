@@ -5,10 +5,15 @@
 A "step" is one leapfrog time step of the whole hot path (SURVEY §8(a) rows
 a2-a6; the once-per-room classification a1 is timed inside `e2e`).  Workload at
 N=1: BASELINE.json configs[3], the C4 hall 1536x1024x704 (1.107e9 voxels), box,
-FD-MM with 3 branches and 8 materials, fp32.  N>1 (torchrun, one rank per GPU):
-weak scaling, the hall grows to 704*N planes, z-slab partitioned
-(rafd_slab_plan), one-plane NCCL halo exchange per step.  Inputs are synthetic
-and seeded (paper_conf_ipps_stoltzfushsld21_b200/inputs.py) and larger than L2.
+FD-MM with 3 branches and 8 materials, fp32; the line also carries
+`single_step` (the same room at one step per sweep: Listings 2-4 iterated) and
+`strong_t1` (C5, configs[4], on one GPU: T_1 of the strong-scaling curve).
+N>1 (torchrun, one rank per GPU): C5 2048x1536x2560 (8.05e9 voxels) split into N
+z-slabs (rafd_slab_plan; strong scaling, E_p = T_1 / (p T_p)), one-plane halo
+exchange per step (NCCL send/recv by default), then a bitwise parity check of
+the slab transport against the CPU oracle (`parity`).  `--config C4` at N>1
+keeps the earlier weak scaling (704*N planes).  Inputs are synthetic and seeded
+(paper_conf_ipps_stoltzfushsld21_b200/inputs.py) and larger than L2.
 
 Prints ONE JSON line on rank 0.  `value` = inside-voxel updates of all ranks /
 max-over-ranks device time (CUDA events on the room's stream).
@@ -19,6 +24,7 @@ import argparse
 import json
 import math
 import os
+import socket
 import subprocess
 import sys
 import threading
@@ -182,8 +188,90 @@ def connect_ipc(room, rank, world, push=False):
     torch.distributed.barrier()
 
 
+def make_room(cfg, prec, rank, world, local_rank, transport, stream, tb_want):
+    """The room (or this rank's slab of it) of a config, inputs generated on
+    the device; temporal blocking enabled as asked (auto: >= 2^25 voxels)."""
+    from paper_conf_ipps_stoltzfushsld21_b200 import rafd
+    dev = torch.device("cuda", local_rank)
+    nx, ny, nz = cfg["room"]
+    beta0, D, E, F = I.config_materials(cfg)
+    plan = slab_plan_box(nx, ny, nz, prec, cfg["MB"], world)
+    z0, z1 = plan[rank]
+    nccl_id = _new_nccl_id(world > 1 and transport == "nccl", rank)
+    mask, mm, mz0 = slab_inputs(cfg, z0, z1, dev)
+    t_c = time.perf_counter()
+    room = rafd.Room(mask, LAM, prec, beta0, D, E, F, matmap=mm, device=local_rank,
+                     stream=None if stream is None else stream.cuda_stream, rank=rank, nranks=world,
+                     nccl_id=nccl_id, z_begin=z0, z_end=z1, mask_z0=mz0, dims=(nx, ny, nz))
+    del mask, mm
+    torch.cuda.empty_cache()
+    # temporal blocking (a slab: edge planes single-step, the interior two-step),
+    # before the IPC blob (it carries the second buffer pair)
+    tb = enable_tb(room, tb_want, world, dev)
+    if world > 1 and transport in ("ipc", "push"):
+        connect_ipc(room, rank, world, push=transport == "push")
+    t_create = time.perf_counter() - t_c
+    mask_np = None if cfg["shape"] == "box" else I.make_mask(cfg["shape"], nx, ny, nz).numpy()
+    room.set_source(I.source_position((nx, ny, nz), mask_np), I.impulse())
+    room.set_receivers(I.receiver_positions((nx, ny, nz), mask_np))
+    return room, tb, t_create, plan
+
+
+def time_room(room, steps, warmup, stream, world, clk=None):
+    """W untimed steps, then K steps between CUDA events on the room's stream
+    (barrier + synchronize on both sides); per-kernel CUDA-event times."""
+    room.step(warmup)
+    room.synchronize()
+    room.read_receivers()
+    room.set_profiling(True)
+    n0 = room.launch_count()
+    ev0 = torch.cuda.Event(enable_timing=True)
+    ev1 = torch.cuda.Event(enable_timing=True)
+    if world > 1:
+        torch.distributed.barrier()
+    torch.cuda.synchronize()
+    import contextlib
+    with (clk if clk is not None else contextlib.nullcontext()):
+        with torch.cuda.stream(stream):
+            ev0.record(stream)
+            room.step(steps)
+            ev1.record(stream)
+        torch.cuda.synchronize()
+    if world > 1:
+        torch.distributed.barrier()
+    ms = ev0.elapsed_time(ev1)
+    launches = room.launch_count() - n0
+    kt = room.get_kernel_times()
+    room.set_profiling(False)
+    rec = room.read_receivers()
+    return ms, launches, kt, rec
+
+
+def sub_record(room, steps, warmup, stream, prec, tb, peak):
+    """One-GPU record of a room at a given steps-per-sweep (the `single_step`
+    and `strong_t1` records of the N=1 line)."""
+    ms, launches, kt, _ = time_room(room, steps, warmup, stream, 1)
+    info = room.get_info()
+    s = prec // 8
+    vol_bytes = info["volume_bytes"] if tb == 1 else info["n_mask"] + info["n_inside"] * 4 * s
+    launch_ms = kt["volume_ms"] / max(1, kt["volume_launches"])
+    bnd_launch_ms = kt["boundary_ms"] / max(1, kt["boundary_launches"])
+    vol_gbs = vol_bytes / (launch_ms * 1e-3) / 1e9
+    return {"value": round(info["n_inside"] * steps / (ms * 1e-3) / 1e9, 3), "unit": UNIT,
+            "ms_per_step": round(ms / steps, 4), "steps": steps, "warmup": warmup, "steps_per_sweep": tb,
+            "n_inside": info["n_inside"],
+            "volume_kernel": "k_volume2 (two steps per sweep)" if tb == 2 else "k_volume_tma",
+            "volume_launch_ms": round(launch_ms, 5), "volume_gbs": round(vol_gbs, 1),
+            "volume_frac_of_peak": round(vol_gbs / peak, 4),
+            "boundary_us_per_launch": round(bnd_launch_ms * 1e3, 2),
+            "boundary_gbs": round(info["boundary_bytes"] / (bnd_launch_ms * 1e-3) / 1e9, 1)
+            if info["n_boundary"] else None,
+            "shell_us_per_step": round(kt["shell_ms"] / steps * 1e3, 2),
+            "gpu_launches": int(launches)}
+
+
 def run_rafd(args, rank, world, local_rank):
-    from paper_conf_ipps_stoltzfushsld21_b200 import build, rafd
+    from paper_conf_ipps_stoltzfushsld21_b200 import build
     if rank == 0:
         build.build()
     if world > 1:
@@ -194,59 +282,11 @@ def run_rafd(args, rank, world, local_rank):
     cfg = workload(args.config, world)
     nx, ny, nz = cfg["room"]
     prec = cfg["precision"] if args.precision is None else args.precision
-    beta0, D, E, F = I.config_materials(cfg)
-    plan = slab_plan_box(nx, ny, nz, prec, cfg["MB"], world)
-    z0, z1 = plan[rank]
-    nccl_id = None
-    if world > 1 and args.transport == "nccl":
-        obj = [rafd.rafd_nccl_unique_id() if rank == 0 else None]
-        torch.distributed.broadcast_object_list(obj, src=0)
-        nccl_id = obj[0]
     stream = torch.cuda.Stream(device=dev)
-    mask, mm, mz0 = slab_inputs(cfg, z0, z1, dev)
-    t_c = time.perf_counter()
-    room = rafd.Room(mask, LAM, prec, beta0, D, E, F, matmap=mm, device=local_rank,
-                     stream=stream.cuda_stream, rank=rank, nranks=world, nccl_id=nccl_id,
-                     z_begin=z0, z_end=z1, mask_z0=mz0, dims=(nx, ny, nz))
-    del mask, mm
-    torch.cuda.empty_cache()
-    # temporal blocking (a slab: edge planes single-step, the interior two-step),
-    # before the IPC blob (it carries the second buffer pair)
-    tb = enable_tb(room, args.tb, world, dev)
-    if world > 1 and args.transport in ("ipc", "push"):
-        connect_ipc(room, rank, world, push=args.transport == "push")
-    t_create = time.perf_counter() - t_c
-    mask_np = None if cfg["shape"] == "box" else I.make_mask(cfg["shape"], nx, ny, nz).numpy()
-    room.set_source(I.source_position((nx, ny, nz), mask_np), I.impulse())
-    room.set_receivers(I.receiver_positions((nx, ny, nz), mask_np))
+    room, tb, t_create, plan = make_room(cfg, prec, rank, world, local_rank, args.transport, stream, args.tb)
     info = room.get_info()
-
-    # warm-up (also builds the CUDA graphs)
-    room.step(args.warmup)
-    room.synchronize()
-    room.read_receivers()
-
     clk = ClockSampler(local_rank)
-    room.set_profiling(True)
-    n0 = room.launch_count()
-    ev0 = torch.cuda.Event(enable_timing=True)
-    ev1 = torch.cuda.Event(enable_timing=True)
-    if world > 1:
-        torch.distributed.barrier()
-    torch.cuda.synchronize()
-    with clk:
-        with torch.cuda.stream(stream):
-            ev0.record(stream)
-            room.step(args.steps)
-            ev1.record(stream)
-        torch.cuda.synchronize()
-    if world > 1:
-        torch.distributed.barrier()
-    ms = ev0.elapsed_time(ev1)
-    launches = room.launch_count() - n0
-    kt = room.get_kernel_times()
-    room.set_profiling(False)
-    rec = room.read_receivers()
+    ms, launches, kt, rec = time_room(room, args.steps, args.warmup, stream, world, clk)
 
     info = room.get_info()
     t = torch.tensor([ms, float(info["n_inside"]), float(info["bytes_per_step"]), float(launches),
@@ -261,10 +301,11 @@ def run_rafd(args, rank, world, local_rank):
     n_in_total = float(sm[1])
     bytes_total = float(sm[2])
     value = n_in_total * args.steps / (ms_max * 1e-3) / 1e9
+    strong = world > 1 and args.config == "C5"
 
     out = None
+    peak, peak_src = peaks()
     if rank == 0:
-        peak, peak_src = peaks()
         fused = bool(info["fused"])
         # per step: one volume launch per step on one GPU; a slab splits it into
         # edge-plane and interior launches, so sum them per step
@@ -285,8 +326,9 @@ def run_rafd(args, rank, world, local_rank):
         vol_gbs = vol_bytes / (launch_ms * 1e-3) / 1e9
         bnd_gbs = info["boundary_bytes"] / (bnd_ms * 1e-3) / 1e9 if (info["n_boundary"] and bnd_ms > 0) else None
         step_gbs = bytes_total * args.steps / (ms_max * 1e-3) / 1e9 / world
-        traffic = None
-        # ncu DRAM bytes of one launch of the timed kernel on this config (committed under profiles/)
+        traffic, traffic_src = None, None
+        # ncu DRAM bytes of one launch of the timed kernel on this config: a
+        # committed `ncu --set full` capture (profiles/), not measured in this run
         tp = os.path.join(ROOT, "profiles", "volume2_traffic.json" if tb == 2 else "volume_traffic.json")
         if os.path.exists(tp):
             try:
@@ -294,12 +336,14 @@ def run_rafd(args, rank, world, local_rank):
                 if bool(tj.get("fused", False)) == fused and args.config == "C4" and world == 1 \
                         and tj.get("precision", 32) == prec:
                     traffic = tj.get("dram_bytes_per_launch")
+                    traffic_src = ("committed constant: ncu --set full capture " + os.path.relpath(tp, ROOT)
+                                   + (f" ({tj['source']})" if tj.get("source") else "") + "; not measured in this run")
             except Exception:
                 traffic = None
         out = {
             "metric": METRIC, "value": round(value, 3), "unit": UNIT, "n_gpus": world,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(ms_max / args.steps, 4),
-            "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
+            "higher_is_better": True, "scaling": "strong" if strong else "weak", "vs_baseline": None,
             "dtype": "f32" if prec == 32 else "f64",
             "data": f"synthetic (seeded {cfg['shape']} room, {cfg['rule']} materials, "
                     + ("seeded FD tables" if cfg['MB'] else "FI admittances from absorption") + ", impulse source)",
@@ -324,6 +368,7 @@ def run_rafd(args, rank, world, local_rank):
                           ("k_volume_tma (volume + fused FD-MM boundary)" if fused else "k_volume_tma"),
                 "achieved": round(vol_gbs, 1), "peak": peak,
                 "unit": "GB/s", "frac": round(vol_gbs / peak, 4), "traffic": traffic,
+                "traffic_source": traffic_src,
                 "algorithmic_bytes_per_launch": vol_bytes,
                 "avg_launch_ms": round(launch_ms, 5), "launches_per_step": kt["volume_launches"] / args.steps,
                 "peak_source": peak_src,
@@ -336,25 +381,127 @@ def run_rafd(args, rank, world, local_rank):
                 "boundary_gbs": None if bnd_gbs is None else round(bnd_gbs, 1),
                 "boundary_share": round(bnd_ms / (ms_max / args.steps), 4),
                 "fused_boundary": fused,
-                # the one-step-per-sweep method's algorithmic bytes (SURVEY §8(d) B_step) per
-                # step over the measured time: > 1 means temporal blocking beats that roofline
-                "step_algorithmic_gbs_per_gpu": round(step_gbs, 1),
-                "step_frac_of_peak": round(step_gbs / peak, 4),
+                # the one-step-per-sweep method's algorithmic bytes (SURVEY §8(d) B_step)
+                # per step over the measured time.  An EQUIVALENT bandwidth, not DRAM
+                # throughput: with two steps per sweep fewer bytes actually move, so
+                # it can exceed the copy peak
+                "step_equivalent_gbs_per_gpu": round(step_gbs, 1),
+                "step_equivalent_frac_of_peak": round(step_gbs / peak, 4),
             },
             "gpu_launches": int(launches),
             "clocks": clk.result(),
             "create_s": round(t_create, 3),
             "receivers_checksum": float(np.abs(rec).sum()),
         }
+    if world == 1 and not args.no_sub_records:
+        # the north_star's two-kernel step (Listings 2-4, one step per sweep),
+        # measured in the same run on the same room
+        if tb == 2:
+            room.set_temporal_blocking(1)
+            out["single_step"] = sub_record(room, args.steps, args.warmup, stream, prec, 1, peak)
+            out["single_step"]["what"] = ("PAPER.md Listings 2-4 iterated (volume kernel + FD-MM boundary "
+                                          "kernel per step, source/receivers fused), same room")
     room.destroy()
     del room
     torch.cuda.synchronize()
     torch.cuda.empty_cache()
-    e2e = run_e2e(args, cfg, prec, beta0, D, E, F, rank, world, local_rank, plan,
+    if world == 1 and args.config == "C4" and not args.no_sub_records:
+        # C5 (BASELINE configs[4]) on one GPU: T_1 of the strong-scaling curve
+        c5 = workload("C5", 1)
+        r5, tb5, _, _ = make_room(c5, prec, 0, 1, local_rank, args.transport, stream, args.tb)
+        rec5 = sub_record(r5, args.steps, args.warmup, stream, prec, tb5, peak)
+        rec5["workload"] = "C5: 2048x1536x2560 box room, FD-MM MB=3 M=8, fp%d, 1 GPU" % prec
+        rec5["efficiency_formula"] = ("E_p = T_1 / (p * T_p), T = ms_per_step of C5: this record (p = 1) and "
+                                      "`bench.py --gpus p` (C5 split into p z-slabs)")
+        out["strong_t1"] = rec5
+        r5.destroy()
+        del r5
+        torch.cuda.synchronize()
+        torch.cuda.empty_cache()
+    e2e = run_e2e(args, cfg, prec, *I.config_materials(cfg), rank, world, local_rank, plan,
                   world > 1 and args.transport == "nccl")
     if rank == 0:
         out["e2e"] = e2e
+    if world > 1:
+        par = parity_leg(args, rank, world, local_rank)
+        if rank == 0:
+            out["parity"] = par
     return out
+
+
+def parity_leg(args, rank, world, local_rank, steps=49):
+    """N > 1 self-check, run after the timing: a small non-cuboid FD-MM room
+    (dome 96 x 80 x 16N, MB=3, M=8, fp32, random initial field, source and
+    receivers) split into the N ranks' z-slabs over the bench's transport,
+    stepped with one and with two steps per sweep; fields, branch state and
+    receivers gathered on rank 0 and compared bit for bit with the CPU oracle
+    (SURVEY §8(c) acceptance)."""
+    from paper_conf_ipps_stoltzfushsld21_b200 import rafd
+    dims = (96, 80, 16 * world)
+    mask_t = I.dome_mask(*dims)
+    mask = mask_t.numpy()
+    mm = I.material_map(mask_t, "region", 8).numpy()
+    beta0, D, E, F = I.fd_tables(8, 3)
+    rng = np.random.default_rng(17)
+    up = (rng.uniform(-1, 1, mask.shape) * mask).astype(np.float32)
+    uc = (rng.uniform(-1, 1, mask.shape) * mask).astype(np.float32)
+    src = I.source_position(dims, mask)
+    rcv = I.receiver_positions(dims, mask)
+    sig = I.gaussian_pulse(40, 4.0)
+    plan = rafd.rafd_slab_plan(mask, 32, 3, world)
+    z0, z1 = plan[rank]
+    res = {"room": "dome %dx%dx%d FD-MM MB=3 M=8 fp32, %d steps" % (dims + (steps,)), "transport": args.transport,
+           "slabs": [list(p) for p in plan]}
+    ref = None
+    if rank == 0:
+        from oracle import orc
+        o = orc.OracleRoom(mask, LAM, 32, beta0, D, E, F, matmap=mm)
+        o.set_state(up, uc)
+        o.set_source(src, sig)
+        o.set_receivers(rcv)
+        o.step(steps)
+        ref = (*o.read_field(), *o.read_branch_state(), o.read_receivers())
+    ok_all = True
+    for tb in (1, 2):
+        nccl_id = _new_nccl_id(args.transport == "nccl", rank)
+        room = rafd.Room(mask, LAM, 32, beta0, D, E, F, matmap=mm, device=local_rank, rank=rank, nranks=world,
+                         nccl_id=nccl_id, z_begin=z0, z_end=z1)
+        room.set_state(up, uc)
+        room.set_source(src, sig)
+        room.set_receivers(rcv)
+        if tb == 2:
+            room.set_temporal_blocking(2)
+        if args.transport in ("ipc", "push"):
+            connect_ipc(room, rank, world, push=args.transport == "push")
+        room.step(steps // 2)
+        room.step(steps - steps // 2)
+        room.synchronize()
+        cur, prv = room.read_field()
+        v, g = room.read_branch_state()
+        rec = room.read_receivers()
+        parts = [None] * world
+        torch.distributed.all_gather_object(parts, (cur, prv, v, g, rec))
+        torch.distributed.barrier()  # IPC: keep the buffers mapped until every neighbour is done
+        room.destroy()
+        if rank == 0:
+            got = (np.concatenate([q[0] for q in parts]), np.concatenate([q[1] for q in parts]),
+                   np.concatenate([q[2] for q in parts], axis=1), np.concatenate([q[3] for q in parts], axis=1),
+                   rafd.gather_receivers([q[4] for q in parts], rcv, plan))
+            eq = [bool(np.array_equal(a, b)) for a, b in zip(got, ref)]
+            res[f"bitwise_tb{tb}"] = dict(zip(["u_n", "u_n_minus_1", "v", "g", "receivers"], eq))
+            ok_all = ok_all and all(eq)
+    if rank == 0:
+        res["parity_ok"] = ok_all
+        log = os.environ.get("NCCL_DEBUG_FILE", "")
+        if log:
+            path = log.replace("%h", socket.gethostname()).replace("%p", str(os.getpid()))
+            try:
+                lines = [ln.strip() for ln in open(path) if "Init COMPLETE" in ln or "nranks" in ln]
+                res["nccl_comm_lines"] = lines[-8:]
+                res["comm_nranks_ok"] = any(f"nranks {world} " in ln for ln in lines)
+            except OSError as e:
+                res["nccl_comm_lines"] = [f"no NCCL debug log ({e})"]
+    return res
 
 
 def enable_tb(room, want, world, dev):
@@ -503,7 +650,27 @@ def oracle_sample(cfg, nplanes):
     return r, (nx, ny, nplanes)
 
 
-def cpu_baseline(cfg, seconds=12.0, nplanes=16):
+def cpu_model():
+    try:
+        for ln in open("/proc/cpuinfo"):
+            if ln.startswith("model name"):
+                return ln.split(":", 1)[1].strip()
+    except OSError:
+        pass
+    import platform
+    return platform.processor() or "unknown"
+
+
+def host_cores():
+    try:
+        return len(os.sched_getaffinity(0))
+    except AttributeError:
+        return os.cpu_count() or 1
+
+
+def _time_oracle(cfg, threads, seconds, nplanes):
+    from oracle import orc
+    orc.set_threads(threads)
     r, dims = oracle_sample(cfg, nplanes)
     n_in = r.info()["n_inside"]
     r.step(1)
@@ -513,16 +680,37 @@ def cpu_baseline(cfg, seconds=12.0, nplanes=16):
         r.step(1)
         n += 1
     dt = time.perf_counter() - t0
-    return {"value": round(n_in * n / dt / 1e9, 5), "unit": UNIT, "cores": 1, "kind": "oracle",
-            "sample": f"{dims[0]}x{dims[1]}x{dims[2]} box crop of the workload (same materials), "
-                      f"{n} steps in {dt:.1f} s, single-threaded C oracle (-O2 -ffp-contract=off)"}
+    return n_in * n / dt / 1e9, n, dt, dims
+
+
+def cpu_baseline(cfg, seconds=8.0):
+    """The oracle as it stands (OpenMP over z planes and boundary nodes, results
+    independent of the thread count) on a bounded sample of the workload: at
+    all host cores (`value`, `cores`) and single-threaded (`single_thread`)."""
+    cores = host_cores()
+    # OpenMP splits the volume loop over z planes: give every thread two planes
+    nplanes = max(16, min(256, 2 * cores))
+    v_n, n_n, dt_n, dims_n = _time_oracle(cfg, cores, seconds, nplanes)
+    v_1, n_1, dt_1, dims_1 = _time_oracle(cfg, 1, seconds, 16)
+    from oracle import orc
+    orc.set_threads(cores)
+    crop = lambda d: f"{d[0]}x{d[1]}x{d[2]} box crop of the workload (same x-y section and materials)"
+    return {"value": round(v_n, 5), "unit": UNIT, "cores": cores, "kind": "oracle",
+            "sample": f"{crop(dims_n)}, {n_n} steps in {dt_n:.1f} s, C oracle (-O2 -ffp-contract=off "
+                      f"-fopenmp, {cores} threads)",
+            "cpu_model": cpu_model(),
+            "single_thread": {"value": round(v_1, 5), "unit": UNIT, "cores": 1,
+                              "sample": f"{crop(dims_1)}, {n_1} steps in {dt_1:.1f} s"}}
 
 
 def run_reference(args):
     """--impl reference: the CPU oracle as it stands (the only reference this
-    tier has), each step a bounded sample of the workload."""
+    tier has) on all host cores, each step a bounded sample of the workload."""
+    from oracle import orc
     cfg = workload(args.config, 1)
-    nplanes = 16
+    cores = host_cores()
+    orc.set_threads(cores)
+    nplanes = max(16, min(256, 2 * cores))
     r, dims = oracle_sample(cfg, nplanes)
     n_in = r.info()["n_inside"]
     r.step(args.warmup)
@@ -536,8 +724,9 @@ def run_reference(args):
             "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
             "dtype": "f32" if cfg["precision"] == 32 else "f64", "data": "synthetic",
             "config": {"workload": f"{args.config} sample: {sample}"},
-            "cpu_baseline": {"value": round(v, 5), "unit": UNIT, "cores": 1, "kind": "oracle",
-                             "sample": sample},
+            "cpu_baseline": {"value": round(v, 5), "unit": UNIT, "cores": cores, "kind": "oracle",
+                             "sample": sample + f", C oracle with OpenMP ({cores} threads)",
+                             "cpu_model": cpu_model()},
             "e2e": {"value": round(v, 5), "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
 
 
@@ -547,9 +736,13 @@ def main():
     ap.add_argument("--steps", type=int, default=200)
     ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--impl", default="rafd", choices=["rafd", "reference"])
-    ap.add_argument("--config", default="C4")
+    ap.add_argument("--config", default=None,
+                    help="default: C4 at N=1 (BASELINE configs[3]); C5 split into N z-slabs at N>1 "
+                         "(configs[4], strong scaling)")
     ap.add_argument("--precision", type=int, default=None)
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-sub-records", action="store_true",
+                    help="N=1: skip the single_step (C4, one step per sweep) and strong_t1 (C5 on one GPU) records")
     ap.add_argument("--tb", type=int, default=0, choices=[0, 1, 2],
                     help="steps per HBM sweep (2: temporal blocking); 0 = auto: 2 for rooms of >= 2^25 "
                          "voxels per GPU, 1 below (measured: C2 256^3 is faster with single steps, C3 and "
@@ -561,8 +754,15 @@ def main():
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local_rank = int(os.environ.get("LOCAL_RANK", "0"))
+    if args.config is None:
+        args.config = "C5" if world > 1 and args.impl != "reference" else "C4"
+    if world > 1 and "NCCL_DEBUG" not in os.environ:
+        # communicator init lines (nranks, devices) for the parity record, in a file:
+        # stdout carries only the JSON line
+        os.environ.update(NCCL_DEBUG="INFO", NCCL_DEBUG_SUBSYS="INIT",
+                          NCCL_DEBUG_FILE="/tmp/rafd_nccl.%h.%p.log")
     if args.impl == "reference":
-        if rank == 0:
+        if rank == 0:  # the oracle is a CPU program: rank 0 alone runs it
             print(json.dumps(run_reference(args)), flush=True)
         return
     if world > 1:

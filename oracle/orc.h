@@ -99,6 +99,10 @@ int  orc_get_info(orc_room *r, orc_info *info);
 /* Discrete energy H^{n+1/2} (reading R11), in double. */
 int  orc_energy(orc_room *r, double *H);
 const char *orc_last_error(void);
+/* OpenMP threads for the volume / boundary loops (process-wide); results are
+ * independent of the count. */
+int  orc_set_threads(int32_t n);
+int32_t orc_get_threads(void);
 
 #ifdef __cplusplus
 }

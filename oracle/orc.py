@@ -17,7 +17,7 @@ _HERE = os.path.dirname(os.path.abspath(__file__))
 _LIB_PATH = os.path.join(_HERE, "liborc.so")
 _SOURCES = ["orc.c", "orc_step.inc", "orc.h"]
 
-CFLAGS = ["-std=c11", "-O2", "-ffp-contract=off", "-fPIC", "-shared", "-Wall", "-Wextra",
+CFLAGS = ["-std=c11", "-O2", "-ffp-contract=off", "-fopenmp", "-fPIC", "-shared", "-Wall", "-Wextra",
           "-Wno-unused-parameter"]
 
 
@@ -70,8 +70,19 @@ def lib():
         L.orc_get_info.argtypes = [P, C.POINTER(OrcInfo)]
         L.orc_energy.argtypes = [P, C.POINTER(C.c_double)]
         L.orc_last_error.restype = C.c_char_p
+        L.orc_set_threads.argtypes = [C.c_int32]
+        L.orc_get_threads.restype = C.c_int32
         _lib = L
     return _lib
+
+
+def set_threads(n: int) -> None:
+    """OpenMP threads of the oracle's volume / boundary loops (process-wide)."""
+    _check(lib().orc_set_threads(int(n)))
+
+
+def get_threads() -> int:
+    return int(lib().orc_get_threads())
 
 
 class OracleError(RuntimeError):

@@ -29,7 +29,9 @@ struct NcclApi {
     ncclResult_t (*GroupStart)() = nullptr;
     ncclResult_t (*GroupEnd)() = nullptr;
     const char *(*GetErrorString)(ncclResult_t) = nullptr;
+    ncclResult_t (*CommGetAsyncError)(ncclComm_t, ncclResult_t *) = nullptr;  // NCCL >= 2.4 (optional)
 };
+static const int ncclInProgress = 7;
 
 static thread_local std::string h_err;
 const char *halo_last_error() { return h_err.c_str(); }
@@ -65,6 +67,7 @@ static NcclApi *api()
     SYM(GroupEnd, "ncclGroupEnd")
     SYM(GetErrorString, "ncclGetErrorString")
 #undef SYM
+    *(void **)(&a.CommGetAsyncError) = dlsym(a.lib, "ncclCommGetAsyncError");
     return &a;
 }
 
@@ -138,6 +141,16 @@ cudaError_t halo_exchange(Halo *h, void *buf, size_t plane_bytes, int lnz, cudaS
     if (r || r2) {
         h_err = std::string("nccl halo exchange: ") + a->GetErrorString(r ? r : r2);
         return cudaErrorUnknown;
+    }
+    // an asynchronous fault (a peer died, a network error) would otherwise
+    // surface only as a hang or wrong ghost planes
+    if (a->CommGetAsyncError) {
+        ncclResult_t ae = 0;
+        ncclResult_t q = a->CommGetAsyncError(h->comm, &ae);
+        if (q != 0 || (ae != 0 && ae != ncclInProgress)) {
+            h_err = std::string("nccl asynchronous error: ") + a->GetErrorString(q ? q : ae);
+            return cudaErrorUnknown;
+        }
     }
     return cudaGetLastError();
 }

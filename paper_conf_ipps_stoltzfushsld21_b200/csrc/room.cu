@@ -1550,29 +1550,67 @@ extern "C" int rafd_get_kernel_times(rafd_room *r, rafd_kernel_times *t)
 extern "C" int64_t rafd_launch_count(rafd_room *r) { return r ? r->launches : 0; }
 
 // ------------------------------------------------------------------ temporal blocking
+// Transactional: the second buffer pair and both new plans are built aside and
+// swapped in only when every step succeeded; on failure the room is left
+// exactly as it was (its single-step plan, graphs and buffers untouched).
 template <typename T> static int enable_twostep_t(rafd_room *r)
 {
-    int rc;
-    const size_t fb = (size_t)r->g.total * sizeof(T) + 64;
-    for (int k = 2; k < 4; k++)
-        if (!r->u[k]) {
-            if ((rc = dmalloc(r, &r->u[k], fb))) return rc;
-            CK(cudaMemsetAsync(r->u[k], 0, fb, r->stream));
-        }
-    if (!r->tbplan) {
-        // the single-step kernel needs TMA maps of the second pair too
-        volume_plan_destroy(r->vplan);
-        r->vplan = nullptr;
-        CK(volume_plan_create<T>(r->g, r->u, r->K_alloc, r->nsm, &r->vplan));
-        const char *sk = getenv("RAFD_SKIP_EMPTY");
-        if (!(sk && strcmp(sk, "0") == 0)) CK(volume_plan_occupancy(r->vplan, r->g, r->K, r->stream));
-        CK(twostep_plan_create<T>(r->g, r->u, r->K_alloc, r->K, r->idx64, r->nsm, r->stream, &r->tbplan, &r->n_shell));
-        r->device_bytes += r->n_shell * (r->idx64 ? 8 : 4) + 56;
-        Ctl<T> c;
-        if ((rc = pull_ctl<T>(r, c))) return rc;
-        CK(twostep_set_source(r->tbplan, c.src_pos, r->g));
+    if (r->tbplan) {
+        CK(cudaStreamSynchronize(r->stream));
+        return RAFD_OK;
     }
-    CK(cudaStreamSynchronize(r->stream));
+    const size_t fb = (size_t)r->g.total * sizeof(T) + 64;
+    void *nu[4] = {r->u[0], r->u[1], r->u[2], r->u[3]};
+    bool fresh[4] = {false, false, false, false};
+    void *vp = nullptr, *tp = nullptr;
+    int64_t nsh = 0;
+    cudaError_t e = cudaSuccess;
+    int rc = RAFD_OK;
+    auto undo = [&]() {
+        cudaStreamSynchronize(r->stream);
+        if (tp) twostep_plan_destroy(tp);
+        if (vp) volume_plan_destroy(vp);
+        for (int k = 2; k < 4; k++)
+            if (fresh[k]) {
+                cudaFree(nu[k]);
+                r->device_bytes -= (int64_t)fb + 64;
+            }
+    };
+    for (int k = 2; k < 4 && rc == RAFD_OK; k++)
+        if (!nu[k]) {
+            if ((rc = dmalloc(r, &nu[k], fb)) == RAFD_OK) {
+                fresh[k] = true;
+                e = cudaMemsetAsync(nu[k], 0, fb, r->stream);
+                if (e != cudaSuccess) rc = -1;
+            }
+        }
+    // the single-step kernel needs TMA maps of the second pair too
+    if (rc == RAFD_OK && e == cudaSuccess) e = volume_plan_create<T>(r->g, nu, r->K_alloc, r->nsm, &vp);
+    const char *sk = getenv("RAFD_SKIP_EMPTY");
+    if (rc == RAFD_OK && e == cudaSuccess && !(sk && strcmp(sk, "0") == 0))
+        e = volume_plan_occupancy(vp, r->g, r->K, r->stream);
+    if (rc == RAFD_OK && e == cudaSuccess)
+        e = twostep_plan_create<T>(r->g, nu, r->K_alloc, r->K, r->idx64, r->nsm, r->stream, &tp, &nsh);
+    Ctl<T> c;
+    if (rc == RAFD_OK && e == cudaSuccess) {
+        if ((rc = pull_ctl<T>(r, c)) == RAFD_OK) e = twostep_set_source(tp, c.src_pos, r->g);
+    }
+    if (rc == RAFD_OK && e == cudaSuccess) e = cudaStreamSynchronize(r->stream);
+    if (rc != RAFD_OK || e != cudaSuccess) {
+        undo();
+        if (rc != RAFD_OK && rc != -1) return rc;
+        cudaGetLastError();
+        return set_err(e == cudaErrorMemoryAllocation ? RAFD_E_NOMEM : RAFD_E_CUDA,
+                       "enabling temporal blocking: %s", cudaGetErrorString(e));
+    }
+    // commit: the cached graphs captured the old plan's arguments
+    free_graphs(r);
+    volume_plan_destroy(r->vplan);
+    r->vplan = vp;
+    r->tbplan = tp;
+    r->n_shell = nsh;
+    r->device_bytes += r->n_shell * (r->idx64 ? 8 : 4) + 56;
+    for (int k = 2; k < 4; k++) r->u[k] = nu[k];
     return RAFD_OK;
 }
 
