@@ -123,8 +123,8 @@ cudaError_t launch_shell(const void *plan, const Grid &g, const T *u1, const T *
 template <typename T>
 cudaError_t launch_boundary(int MB, bool idx64, const void *bpos, const uint8_t *Kb,
                             const uint8_t *matb, int64_t i_lo, int64_t i_hi, int64_t Nb, T *unext,
-                            T *ub, T *g, T *v, const T *tab, int M, double lambda, cudaStream_t s,
-                            int64_t mirror0 = 0, int64_t mirror1 = 0, Ctl<T> *ctl = nullptr,
+                            T *ub, T *g, T *v, const T *tab, const T *tab_host, int M, double lambda,
+                            cudaStream_t s, int64_t mirror0 = 0, int64_t mirror1 = 0, Ctl<T> *ctl = nullptr,
                             unsigned int *ticket = nullptr, int src_mode = 3);
 template <typename T>
 cudaError_t launch_src_rcv(T *unext, T *ub, Ctl<T> *ctl, cudaStream_t s, int mode = 3, int64_t mirror0 = 0,

@@ -109,6 +109,7 @@ struct rafd_room {
     uint8_t *Kb = nullptr, *matb = nullptr;
     void *ub = nullptr, *gst = nullptr, *vst = nullptr;
     void *tab = nullptr;   // T: beta[M] | BI | D | DI | F  ([M*MB] each)
+    std::vector<unsigned char> tab_host;  // the same table on the host (boundary-kernel launch parameter)
     double *DF = nullptr;  // double D | F for the energy hook
     void *ctl = nullptr;   // Ctl<T>
     unsigned int *ticket = nullptr;  // last-block ticket of the boundary kernel's fused source/receivers
@@ -415,6 +416,7 @@ template <typename T> static int create_t(rafd_room *r, const rafd_room_desc *d)
     if ((rc = dmalloc(r, &r->tab, tab.size() * sizeof(T)))) return rc;
     if ((rc = dmalloc(r, (void **)&r->DF, DF.size() * sizeof(double)))) return rc;
     CK(cudaMemcpy(r->tab, tab.data(), tab.size() * sizeof(T), cudaMemcpyHostToDevice));
+    r->tab_host.assign((const unsigned char *)tab.data(), (const unsigned char *)(tab.data() + tab.size()));
     CK(cudaMemcpy(r->DF, DF.data(), DF.size() * sizeof(double), cudaMemcpyHostToDevice));
     if ((rc = dmalloc(r, &r->ctl, sizeof(Ctl<T>)))) return rc;
     if ((rc = dmalloc(r, (void **)&r->ticket, sizeof(unsigned int)))) return rc;
@@ -739,7 +741,7 @@ template <typename T> static cudaError_t enqueue_step(rafd_room *r, int pair, in
         // the source and receivers run in the boundary kernel's last block
         return timed(1, [&] {
             return launch_boundary<T>(r->MB, r->idx64, r->bpos, r->Kb, r->matb, 0, r->nb, r->nb, un,
-                                      ub_slot<T>(r, cur), (T *)r->gst, (T *)r->vst, (const T *)r->tab, r->M,
+                                      ub_slot<T>(r, cur), (T *)r->gst, (T *)r->vst, (const T *)r->tab, (const T *)r->tab_host.data(), r->M,
                                       r->lambda, s, 0, 0, ctl_of<T>(r), r->ticket);
         });
     }
@@ -762,7 +764,7 @@ template <typename T> static cudaError_t enqueue_step2(rafd_room *r, int pair, i
             return timed_launch(r, s, prof, 2, [&] { return launch_src_rcv<T>(un, ub_slot<T>(r, slot), ctl_of<T>(r), s); });
         return timed_launch(r, s, prof, 1, [&] {
             return launch_boundary<T>(r->MB, r->idx64, r->bpos, r->Kb, r->matb, 0, r->nb, r->nb, un,
-                                      ub_slot<T>(r, slot), (T *)r->gst, (T *)r->vst, (const T *)r->tab, r->M,
+                                      ub_slot<T>(r, slot), (T *)r->gst, (T *)r->vst, (const T *)r->tab, (const T *)r->tab_host.data(), r->M,
                                       r->lambda, s, 0, 0, ctl_of<T>(r), r->ticket);
         });
     };
@@ -805,7 +807,7 @@ static cudaError_t enqueue_phase(rafd_room *r, int phase, cudaStream_t s, bool p
         if (hi <= lo || r->fused || r->scheme) return cudaSuccess;
         return timed(1, [&] {
             return launch_boundary<T>(r->MB, r->idx64, r->bpos, r->Kb, r->matb, lo, hi, r->nb, un,
-                                      ub_slot<T>(r, cur), (T *)r->gst, (T *)r->vst, (const T *)r->tab, r->M,
+                                      ub_slot<T>(r, cur), (T *)r->gst, (T *)r->vst, (const T *)r->tab, (const T *)r->tab_host.data(), r->M,
                                       r->lambda, s, m0, m1, src_mode ? ctl_of<T>(r) : nullptr, r->ticket,
                                       src_mode);
         });
@@ -893,7 +895,7 @@ static cudaError_t enqueue_tb_phase(rafd_room *r, int ph, cudaStream_t s, bool p
         if (hi <= lo) return cudaSuccess;
         return timed(1, [&] {
             return launch_boundary<T>(r->MB, r->idx64, r->bpos, r->Kb, r->matb, lo, hi, r->nb, out, ub, (T *)r->gst,
-                                      (T *)r->vst, (const T *)r->tab, r->M, r->lambda, s, m0, m1,
+                                      (T *)r->vst, (const T *)r->tab, (const T *)r->tab_host.data(), r->M, r->lambda, s, m0, m1,
                                       src_mode ? ctl_of<T>(r) : nullptr, r->ticket, src_mode);
         });
     };
