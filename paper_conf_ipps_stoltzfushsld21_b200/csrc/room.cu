@@ -29,6 +29,26 @@ using namespace rafd;
 // ------------------------------------------------------------------ errors
 static thread_local std::string g_err;
 
+// Setup-phase tracing (RAFD_TRACE=1): synchronises the room's stream at each
+// mark and prints the wall time of the phase to stderr.  Off: one branch.
+#include <chrono>
+struct PhaseTrace {
+    bool on;
+    std::chrono::steady_clock::time_point t;
+    explicit PhaseTrace(const char *what) : on(getenv("RAFD_TRACE") != nullptr), t(std::chrono::steady_clock::now())
+    {
+        if (on) fprintf(stderr, "[rafd] %s\n", what);
+    }
+    void mark(cudaStream_t s, const char *name)
+    {
+        if (!on) return;
+        cudaStreamSynchronize(s);
+        const auto n = std::chrono::steady_clock::now();
+        fprintf(stderr, "[rafd]   %-28s %8.2f ms\n", name, std::chrono::duration<double, std::milli>(n - t).count());
+        t = n;
+    }
+};
+
 static int set_err(int code, const char *fmt, ...)
 {
     char buf[512];
@@ -305,6 +325,7 @@ template <typename T> static int create_t(rafd_room *r, const rafd_room_desc *d)
     r->idx64 = g.total >= (int64_t)UINT32_MAX;
 
     int rc;
+    PhaseTrace tr("rafd_create");
     // K grid: element (row, xo + x) must sit at a 16-byte aligned byte address
     // for the TMA boxes of the volume kernel, so the buffer starts k_shift(g)
     // bytes before the first element (r->K_alloc is what cudaMalloc returned).
@@ -312,8 +333,10 @@ template <typename T> static int create_t(rafd_room *r, const rafd_room_desc *d)
     r->K = r->K_alloc + k_shift(g);
     for (int k = 0; k < 2; k++)
         if ((rc = dmalloc(r, &r->u[k], (size_t)g.total * sizeof(T) + 64))) return rc;
+    tr.mark(r->stream, "alloc K, u[2]");
     CK(cudaMemsetAsync(r->K_alloc, 0, (size_t)g.total + 64, r->stream));
     for (int k = 0; k < 2; k++) CK(cudaMemsetAsync(r->u[k], 0, (size_t)g.total * sizeof(T) + 64, r->stream));
+    tr.mark(r->stream, "memset K, u[2]");
 
     // ---- classification (row a1)
     // the mask is streamed in full (DMA staging beats zero-copy reads for it);
@@ -331,6 +354,7 @@ template <typename T> static int create_t(rafd_room *r, const rafd_room_desc *d)
                               return RAFD_OK;
                           });
     if (rc) return rc;
+    tr.mark(r->stream, "mask H2D + scatter");
     CK(launch_count_k(g, r->K, r->stream));
     unsigned long long *hist = nullptr;
     if ((rc = dmalloc(r, (void **)&hist, 8 * sizeof(unsigned long long) + sizeof(unsigned)))) return rc;
@@ -354,6 +378,7 @@ template <typename T> static int create_t(rafd_room *r, const rafd_room_desc *d)
     CK(cudaMemcpyAsync(&r->n_first_plane, row_off + std::min<int64_t>(rows, r->ny), 8, cudaMemcpyDeviceToHost, r->stream));
     CK(cudaMemcpyAsync(&r->n_last_start, row_off + (int64_t)(g.lnz - 1) * r->ny, 8, cudaMemcpyDeviceToHost, r->stream));
     CK(cudaStreamSynchronize(r->stream));
+    tr.mark(r->stream, "K, histogram, row scan");
     r->isolated = (int64_t)h[0];
     int64_t nin = 0;
     for (int k = 1; k <= 6; k++) {
@@ -375,6 +400,7 @@ template <typename T> static int create_t(rafd_room *r, const rafd_room_desc *d)
     CK(cudaMemsetAsync(r->gst, 0, (size_t)nb * r->MB * sizeof(T) + 16, r->stream));
     CK(cudaMemsetAsync(r->vst, 0, (size_t)nb * r->MB * sizeof(T) + 16, r->stream));
     CK(launch_compact(g, r->K, row_off, r->z0, r->ny, r->nx, r->idx64, r->bpos, r->bidx, r->Kb, r->stream));
+    tr.mark(r->stream, "boundary SoA alloc + compact");
 
     // material ids at the boundary nodes (reading R4)
     unsigned *bad = (unsigned *)(hist + 8);
@@ -398,6 +424,7 @@ template <typename T> static int create_t(rafd_room *r, const rafd_room_desc *d)
         if (rc) return rc;
     }
     unsigned bad_h = 0;
+    tr.mark(r->stream, "material gather");
     CK(cudaMemcpyAsync(&bad_h, bad, sizeof bad_h, cudaMemcpyDeviceToHost, r->stream));
     CK(cudaStreamSynchronize(r->stream));
     cudaFree(hist);
@@ -425,12 +452,14 @@ template <typename T> static int create_t(rafd_room *r, const rafd_room_desc *d)
     c.src_pos = -1;
     c.src_node = -1;
     CK(cudaMemcpy(r->ctl, &c, sizeof c, cudaMemcpyHostToDevice));
+    tr.mark(r->stream, "tables, control block");
     const char *env = getenv("RAFD_VOLUME_KERNEL");
     if (!(env && strcmp(env, "v0") == 0)) {
         CK(volume_plan_create<T>(g, r->u, r->K_alloc, r->nsm, &r->vplan));
         const char *sk = getenv("RAFD_SKIP_EMPTY");  // skipping of all-outside tile-planes (default on)
         if (!(sk && strcmp(sk, "0") == 0)) CK(volume_plan_occupancy(r->vplan, g, r->K, r->stream));
     }
+    tr.mark(r->stream, "volume plan");
     // boundary update fused into the volume kernel with RAFD_FUSED=1 (DESIGN.md
     // §6; needs the default tiling, MB <= 4, Nb < 2^31).  Off by default: the
     // first fused form is latency-bound at x-wall rows (5.6 ms vs 2.55 ms).
@@ -529,6 +558,7 @@ extern "C" void rafd_destroy(rafd_room *r)
     if (!r) return;
     cudaSetDevice(r->device);
     if (r->stream) cudaStreamSynchronize(r->stream);
+    PhaseTrace tr("rafd_destroy");
     free_graphs(r);
     if (r->halo) halo_destroy(r->halo);
     if (r->ipc) ipc_close(r->ipc);
@@ -542,6 +572,7 @@ extern "C" void rafd_destroy(rafd_room *r)
                   r->tab, r->DF, r->ctl, r->ticket, r->sig, r->rcv_pos, r->rec};
     for (void *p : ps)
         if (p) cudaFree(p);
+    tr.mark(r->stream, "free device buffers");
     for (auto &e : r->evs) {
         cudaEventDestroy(e.a);
         cudaEventDestroy(e.b);
@@ -1578,6 +1609,7 @@ template <typename T> static int enable_twostep_t(rafd_room *r)
                 r->device_bytes -= (int64_t)fb + 64;
             }
     };
+    PhaseTrace tr("rafd_set_temporal_blocking(2)");
     for (int k = 2; k < 4 && rc == RAFD_OK; k++)
         if (!nu[k]) {
             if ((rc = dmalloc(r, &nu[k], fb)) == RAFD_OK) {
@@ -1586,13 +1618,16 @@ template <typename T> static int enable_twostep_t(rafd_room *r)
                 if (e != cudaSuccess) rc = -1;
             }
         }
+    tr.mark(r->stream, "alloc + memset u[2..3]");
     // the single-step kernel needs TMA maps of the second pair too
     if (rc == RAFD_OK && e == cudaSuccess) e = volume_plan_create<T>(r->g, nu, r->K_alloc, r->nsm, &vp);
     const char *sk = getenv("RAFD_SKIP_EMPTY");
     if (rc == RAFD_OK && e == cudaSuccess && !(sk && strcmp(sk, "0") == 0))
         e = volume_plan_occupancy(vp, r->g, r->K, r->stream);
+    tr.mark(r->stream, "volume plan");
     if (rc == RAFD_OK && e == cudaSuccess)
         e = twostep_plan_create<T>(r->g, nu, r->K_alloc, r->K, r->idx64, r->nsm, r->stream, &tp, &nsh);
+    tr.mark(r->stream, "two-step plan + shell list");
     Ctl<T> c;
     if (rc == RAFD_OK && e == cudaSuccess) {
         if ((rc = pull_ctl<T>(r, c)) == RAFD_OK) e = twostep_set_source(tp, c.src_pos, r->g);

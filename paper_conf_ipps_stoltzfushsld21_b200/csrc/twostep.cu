@@ -356,72 +356,8 @@ __global__ void __launch_bounds__(TbGeom<T, TY, SU, SP>::NT, 1)
 }
 
 // ------------------------------------------------------------------ the shell
-// shell voxel: inside, and itself or a face neighbour a boundary node
-static __device__ __forceinline__ bool is_shell(const uint8_t *K, int64_t i, const Grid &g)
-{
-    const int k = K[i];
-    if (k == 0) return false;
-    if (k < 6) return true;
-    return K[i - 1] < 6 || K[i + 1] < 6 || K[i - g.pitch] < 6 || K[i + g.pitch] < 6 || K[i - g.plane] < 6 ||
-           K[i + g.plane] < 6;
-}
-
-// per-row counts with a block reduction (one block per row)
-__global__ void k_shell_row_counts(Grid g, const uint8_t *__restrict__ K, int64_t *__restrict__ cnt)
-{
-    __shared__ int red[32];
-    const int64_t rows = (int64_t)g.lnz * g.ny;
-    for (int64_t row = blockIdx.x; row < rows; row += gridDim.x) {
-        const int64_t y = row % g.ny, z = row / g.ny;
-        const int64_t b = (z + 1) * g.plane + (y + 1) * g.pitch + g.xo;
-        int c = 0;
-        for (int x = threadIdx.x; x < g.nx; x += blockDim.x) c += is_shell(K, b + x, g);
-#pragma unroll
-        for (int o = 16; o; o >>= 1) c += __shfl_xor_sync(0xffffffffu, c, o);
-        if ((threadIdx.x & 31) == 0) red[threadIdx.x >> 5] = c;
-        __syncthreads();
-        if (threadIdx.x == 0) {
-            int s = 0;
-            for (int w = 0; w < (int)(blockDim.x >> 5); w++) s += red[w];
-            cnt[row] = s;
-        }
-        __syncthreads();
-    }
-}
-
-// ascending padded positions of the shell voxels (one block per row, a block
-// scan keeps the x order)
-template <typename IdxT>
-__global__ void k_shell_compact(Grid g, const uint8_t *__restrict__ K, const int64_t *__restrict__ off,
-                                IdxT *__restrict__ list)
-{
-    __shared__ int wsum[32];
-    __shared__ int64_t base_s;
-    const int64_t rows = (int64_t)g.lnz * g.ny;
-    const int nwarps = blockDim.x >> 5, lane = threadIdx.x & 31, w = threadIdx.x >> 5;
-    for (int64_t row = blockIdx.x; row < rows; row += gridDim.x) {
-        const int64_t y = row % g.ny, z = row / g.ny;
-        const int64_t b = (z + 1) * g.plane + (y + 1) * g.pitch + g.xo;
-        if (threadIdx.x == 0) base_s = off[row];
-        __syncthreads();
-        for (int x0 = 0; x0 < g.nx; x0 += blockDim.x) {
-            const int x = x0 + threadIdx.x;
-            const bool f = x < g.nx && is_shell(K, b + x, g);
-            const unsigned m = __ballot_sync(0xffffffffu, f);
-            if (lane == 0) wsum[w] = __popc(m);
-            __syncthreads();
-            int before = 0, total = 0;
-            for (int k = 0; k < nwarps; k++) {
-                before += k < w ? wsum[k] : 0;
-                total += wsum[k];
-            }
-            if (f) list[base_s + before + __popc(m & ((1u << lane) - 1u))] = (IdxT)(b + x);
-            __syncthreads();
-            if (threadIdx.x == 0) base_s += total;
-            __syncthreads();
-        }
-    }
-}
+// (the list -- inside voxels that are, or have a face neighbour that is, a
+// boundary node -- is built by classify.cu's row compaction)
 
 // u^{n+2} at the shell voxels and the source's 7-point star (src[7], -1 =
 // none), from the final u^{n+1} (u1) and u^n (u0): the volume update in the
@@ -554,11 +490,7 @@ cudaError_t twostep_plan_create(const Grid &g, void *const u[4], uint8_t *K_allo
     if (e == cudaSuccess) e = cudaMalloc(&cnt, (size_t)(rows + 1) * 8);
     if (e == cudaSuccess) e = cudaMalloc(&off, (size_t)(rows + 1) * 8);
     if (e == cudaSuccess) e = cudaMemsetAsync(cnt, 0, (size_t)(rows + 1) * 8, s);
-    const unsigned blocks = (unsigned)std::max<int64_t>(1, std::min<int64_t>(rows, (int64_t)nsm * 16));
-    if (e == cudaSuccess && rows > 0) {
-        k_shell_row_counts<<<blocks, 256, 0, s>>>(g, K, cnt);
-        e = cudaGetLastError();
-    }
+    if (e == cudaSuccess) e = launch_shell_counts(g, K, cnt, s);
     if (e == cudaSuccess) e = exclusive_scan_rows64(cnt, off, rows + 1, nullptr, &tb, s);
     if (e == cudaSuccess) e = cudaMalloc(&tmp, tb ? tb : 16);
     if (e == cudaSuccess) e = exclusive_scan_rows64(cnt, off, rows + 1, tmp, &tb, s);
@@ -569,11 +501,7 @@ cudaError_t twostep_plan_create(const Grid &g, void *const u[4], uint8_t *K_allo
         e = cudaMemcpyAsync(&pl->sh_hi, off + (int64_t)(g.lnz - 1) * g.ny, 8, cudaMemcpyDeviceToHost, s);
     if (e == cudaSuccess) e = cudaStreamSynchronize(s);
     if (e == cudaSuccess) e = cudaMalloc(&pl->list, (size_t)std::max<int64_t>(n, 1) * (idx64 ? 8 : 4));
-    if (e == cudaSuccess && rows > 0 && n > 0) {
-        if (idx64) k_shell_compact<int64_t><<<blocks, 256, 0, s>>>(g, K, off, (int64_t *)pl->list);
-        else k_shell_compact<uint32_t><<<blocks, 256, 0, s>>>(g, K, off, (uint32_t *)pl->list);
-        e = cudaGetLastError();
-    }
+    if (e == cudaSuccess && n > 0) e = launch_shell_compact(g, K, off, idx64, pl->list, s);
     if (e == cudaSuccess) e = cudaMalloc(&pl->work, 2 * sizeof(unsigned int));
     if (e == cudaSuccess) e = cudaMemsetAsync(pl->work, 0, 2 * sizeof(unsigned int), s);
     if (e == cudaSuccess) e = cudaMalloc(&pl->src, 7 * 8);
