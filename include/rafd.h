@@ -281,6 +281,17 @@ int64_t rafd_launch_count(rafd_room *r);
 int rafd_slab_plan(int32_t nx, int32_t ny, int32_t nz, const uint8_t *mask, int32_t precision,
                    int32_t n_branches, int32_t nranks, int32_t *z_begin, int32_t *z_end);
 
+/* Device memory.  Whole-room handles (nranks <= 1) take their buffers from a
+ * per-device cache owned by the library (a caching allocator over cudaMalloc):
+ * rafd_destroy returns them to the cache (which then keeps at most half of the
+ * device's memory) instead of freeing them, and the next room of a similar
+ * size reuses them.  This call frees every cached block of `device`, e.g.
+ * before another library allocates large buffers (like
+ * torch.cuda.empty_cache()).  Waits for the device.  Rooms still alive keep
+ * their memory.  INVAL (device < 0), CUDA.  Environment RAFD_POOL=0 makes
+ * rooms use cudaMalloc / cudaFree directly. */
+int rafd_release_cached_memory(int32_t device);
+
 /* 128-byte NCCL unique id for a multi-GPU room (call on rank 0, broadcast). */
 int rafd_nccl_unique_id(uint8_t *id128);
 

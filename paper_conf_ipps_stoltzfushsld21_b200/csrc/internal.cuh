@@ -66,6 +66,13 @@ struct KernelTimes {
     int64_t volume_n = 0, boundary_n = 0, other_n = 0, shell_n = 0;
 };
 
+// ------------------------------------------------------------------ device memory (devmem.cu)
+// cached = true: the block may come from / return to the library's cache
+cudaError_t dev_alloc(void **p, size_t bytes, bool cached = true);
+void dev_free(void *p);
+bool dev_cache_enabled();
+void dev_cache_trim(int dev, size_t keep);
+
 // ------------------------------------------------------------------ launchers
 // (each returns cudaGetLastError() of its launch)
 // Arguments of the fused volume+boundary kernel (seg_first is set by the plan).

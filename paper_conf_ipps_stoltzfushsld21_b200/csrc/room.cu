@@ -130,6 +130,7 @@ struct rafd_room {
     void *ub = nullptr, *gst = nullptr, *vst = nullptr;
     void *tab = nullptr;   // T: beta[M] | BI | D | DI | F  ([M*MB] each)
     std::vector<unsigned char> tab_host;  // the same table on the host (boundary-kernel launch parameter)
+    bool use_pool = false;                // buffers through the library's memory cache (whole rooms)
     double *DF = nullptr;  // double D | F for the energy hook
     void *ctl = nullptr;   // Ctl<T>
     unsigned int *ticket = nullptr;  // last-block ticket of the boundary kernel's fused source/receivers
@@ -204,11 +205,15 @@ template <typename T> static FusedArgs<T> fused_args(const rafd_room *r)
     return f;
 }
 
+// ------------------------------------------------------------------ device memory
+// Whole-room handles allocate through the library's cache (devmem.cu); slab
+// handles (nranks > 1) with plain cudaMalloc, since their field buffers may be
+// exported with CUDA IPC.
 // every allocation carries 64 bytes of slack (vector loads / memsets of +16)
 static int dmalloc(rafd_room *r, void **p, size_t bytes)
 {
     bytes += 64;
-    cudaError_t e = cudaMalloc(p, bytes);
+    cudaError_t e = dev_alloc(p, bytes, r->use_pool);
     if (e != cudaSuccess) {
         cudaGetLastError();
         *p = nullptr;
@@ -216,6 +221,14 @@ static int dmalloc(rafd_room *r, void **p, size_t bytes)
     }
     r->device_bytes += (int64_t)bytes;
     return RAFD_OK;
+}
+
+// frees what dmalloc or cudaMalloc returned, once the room's work is done
+static void dfree(rafd_room *r, void *p)
+{
+    if (!p) return;
+    cudaStreamSynchronize(r->stream);
+    dev_free(p);
 }
 
 // ------------------------------------------------------------------ validation
@@ -427,11 +440,11 @@ template <typename T> static int create_t(rafd_room *r, const rafd_room_desc *d)
     tr.mark(r->stream, "material gather");
     CK(cudaMemcpyAsync(&bad_h, bad, sizeof bad_h, cudaMemcpyDeviceToHost, r->stream));
     CK(cudaStreamSynchronize(r->stream));
-    cudaFree(hist);
-    cudaFree(counts);
-    cudaFree(row_off);
-    cudaFree(tmp);
-    if (staging) cudaFree(staging);
+    dfree(r, hist);
+    dfree(r, counts);
+    dfree(r, row_off);
+    dfree(r, tmp);
+    dfree(r, staging);
     r->device_bytes -= (int64_t)(8 * sizeof(unsigned long long) + sizeof(unsigned)) + 2 * (rows + 1) * 8 +
                        (int64_t)(tmpb ? tmpb : 16) + (staging ? (int64_t)kStagingBytes : 0);
     if (bad_h) return set_err(RAFD_E_MATERIAL, "matmap holds a material id >= n_materials (%d) at a boundary node", r->M);
@@ -509,6 +522,7 @@ extern "C" int rafd_create(const rafd_room_desc *d, rafd_room **out)
     r->nranks = d->nranks > 1 ? d->nranks : 1;
     r->z0 = r->nranks > 1 ? d->z_begin : 0;
     r->z1 = r->nranks > 1 ? d->z_end : d->nz;
+    r->use_pool = r->nranks == 1 && dev_cache_enabled();
     cudaDeviceGetAttribute(&r->nsm, cudaDevAttrMultiProcessorCount, r->device);
     if (d->cuda_stream) {
         r->stream = (cudaStream_t)d->cuda_stream;
@@ -570,8 +584,7 @@ extern "C" void rafd_destroy(rafd_room *r)
     if (r->tbplan) twostep_plan_destroy(r->tbplan);
     void *ps[] = {r->u[0], r->u[1], r->u[2], r->u[3], r->K_alloc, r->bpos, r->bidx, r->Kb, r->matb, r->ub, r->gst, r->vst,
                   r->tab, r->DF, r->ctl, r->ticket, r->sig, r->rcv_pos, r->rec};
-    for (void *p : ps)
-        if (p) cudaFree(p);
+    for (void *p : ps) dfree(r, p);
     tr.mark(r->stream, "free device buffers");
     for (auto &e : r->evs) {
         cudaEventDestroy(e.a);
@@ -581,8 +594,21 @@ extern "C" void rafd_destroy(rafd_room *r)
     if (r->rec_host) cudaFreeHost(r->rec_host);
     if (r->cap_stream) cudaStreamDestroy(r->cap_stream);
     if (r->own_stream && r->stream) cudaStreamDestroy(r->stream);
+    if (r->use_pool) {  // keep at most half of the device memory cached
+        size_t fr = 0, tot = 0;
+        if (cudaMemGetInfo(&fr, &tot) == cudaSuccess) dev_cache_trim(r->device, tot / 2);
+    }
     cudaGetLastError();
     delete r;
+}
+
+extern "C" int rafd_release_cached_memory(int32_t device)
+{
+    if (device < 0) return set_err(RAFD_E_INVAL, "device must be >= 0");
+    CK(cudaSetDevice(device));
+    CK(cudaDeviceSynchronize());
+    dev_cache_trim(device, 0);
+    return RAFD_OK;
 }
 
 // ------------------------------------------------------------------ source / receivers
@@ -1605,7 +1631,7 @@ template <typename T> static int enable_twostep_t(rafd_room *r)
         if (vp) volume_plan_destroy(vp);
         for (int k = 2; k < 4; k++)
             if (fresh[k]) {
-                cudaFree(nu[k]);
+                dfree(r, nu[k]);
                 r->device_bytes -= (int64_t)fb + 64;
             }
     };

@@ -487,12 +487,12 @@ cudaError_t twostep_plan_create(const Grid &g, void *const u[4], uint8_t *K_allo
     int64_t *cnt = nullptr, *off = nullptr;
     void *tmp = nullptr;
     size_t tb = 0;
-    if (e == cudaSuccess) e = cudaMalloc(&cnt, (size_t)(rows + 1) * 8);
-    if (e == cudaSuccess) e = cudaMalloc(&off, (size_t)(rows + 1) * 8);
+    if (e == cudaSuccess) e = dev_alloc((void **)&cnt, (size_t)(rows + 1) * 8);
+    if (e == cudaSuccess) e = dev_alloc((void **)&off, (size_t)(rows + 1) * 8);
     if (e == cudaSuccess) e = cudaMemsetAsync(cnt, 0, (size_t)(rows + 1) * 8, s);
     if (e == cudaSuccess) e = launch_shell_counts(g, K, cnt, s);
     if (e == cudaSuccess) e = exclusive_scan_rows64(cnt, off, rows + 1, nullptr, &tb, s);
-    if (e == cudaSuccess) e = cudaMalloc(&tmp, tb ? tb : 16);
+    if (e == cudaSuccess) e = dev_alloc((void **)&tmp, tb ? tb : 16);
     if (e == cudaSuccess) e = exclusive_scan_rows64(cnt, off, rows + 1, tmp, &tb, s);
     int64_t n = 0;
     if (e == cudaSuccess) e = cudaMemcpyAsync(&n, off + rows, 8, cudaMemcpyDeviceToHost, s);
@@ -500,21 +500,21 @@ cudaError_t twostep_plan_create(const Grid &g, void *const u[4], uint8_t *K_allo
     if (e == cudaSuccess && g.lnz >= 2)
         e = cudaMemcpyAsync(&pl->sh_hi, off + (int64_t)(g.lnz - 1) * g.ny, 8, cudaMemcpyDeviceToHost, s);
     if (e == cudaSuccess) e = cudaStreamSynchronize(s);
-    if (e == cudaSuccess) e = cudaMalloc(&pl->list, (size_t)std::max<int64_t>(n, 1) * (idx64 ? 8 : 4));
+    if (e == cudaSuccess) e = dev_alloc((void **)&pl->list, (size_t)std::max<int64_t>(n, 1) * (idx64 ? 8 : 4));
     if (e == cudaSuccess && n > 0) e = launch_shell_compact(g, K, off, idx64, pl->list, s);
-    if (e == cudaSuccess) e = cudaMalloc(&pl->work, 2 * sizeof(unsigned int));
+    if (e == cudaSuccess) e = dev_alloc((void **)&pl->work, 2 * sizeof(unsigned int));
     if (e == cudaSuccess) e = cudaMemsetAsync(pl->work, 0, 2 * sizeof(unsigned int), s);
-    if (e == cudaSuccess) e = cudaMalloc(&pl->src, 7 * 8);
+    if (e == cudaSuccess) e = dev_alloc((void **)&pl->src, 7 * 8);
     if (e == cudaSuccess) e = cudaMemsetAsync(pl->src, 0xff, 7 * 8, s);
     if (e == cudaSuccess) e = cudaStreamSynchronize(s);
-    if (cnt) cudaFree(cnt);
-    if (off) cudaFree(off);
-    if (tmp) cudaFree(tmp);
+    if (cnt) dev_free(cnt);
+    if (off) dev_free(off);
+    if (tmp) dev_free(tmp);
     pl->n_shell = n;
     if (e != cudaSuccess) {
-        if (pl->list) cudaFree(pl->list);
-        if (pl->src) cudaFree(pl->src);
-        if (pl->work) cudaFree(pl->work);
+        if (pl->list) dev_free(pl->list);
+        if (pl->src) dev_free(pl->src);
+        if (pl->work) dev_free(pl->work);
         delete pl;
         return e;
     }
@@ -527,9 +527,9 @@ void twostep_plan_destroy(void *plan)
 {
     auto *pl = (TwoStepPlan *)plan;
     if (!pl) return;
-    if (pl->list) cudaFree(pl->list);
-    if (pl->src) cudaFree(pl->src);
-    if (pl->work) cudaFree(pl->work);
+    if (pl->list) dev_free(pl->list);
+    if (pl->src) dev_free(pl->src);
+    if (pl->work) dev_free(pl->work);
     delete pl;
 }
 

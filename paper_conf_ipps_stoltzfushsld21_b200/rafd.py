@@ -40,7 +40,7 @@ ABI_SYMBOLS = [
     "rafd_set_profiling", "rafd_get_kernel_times", "rafd_launch_count", "rafd_slab_plan",
     "rafd_nccl_unique_id", "rafd_last_error", "rafd_strerror", "rafd_version",
     "rafd_ipc_handle", "rafd_ipc_connect", "rafd_set_step", "rafd_set_temporal_blocking",
-    "rafd_set_halo_push",
+    "rafd_set_halo_push", "rafd_release_cached_memory",
 ]
 RAFD_IPC_BLOB_BYTES = 352
 
@@ -119,6 +119,7 @@ def lib():
     L.rafd_ipc_handle.argtypes = [P, P]
     L.rafd_ipc_connect.argtypes = [P, P, P]
     L.rafd_set_halo_push.argtypes = [P, I32]
+    L.rafd_release_cached_memory.argtypes = [I32]
     L.rafd_last_error.restype = C.c_char_p
     L.rafd_strerror.restype = C.c_char_p
     L.rafd_strerror.argtypes = [C.c_int]
@@ -369,6 +370,11 @@ def gather_receivers(per_slab, xyzs, plan):
     for j, (x, y, z) in enumerate(xyzs):
         out[j] = per_slab[slab_owner(z, plan)][j]
     return out
+
+
+def rafd_release_cached_memory(device=0):
+    """Return the library pool's cached device memory to the driver."""
+    _check(lib().rafd_release_cached_memory(int(device)))
 
 
 def rafd_nccl_unique_id():
