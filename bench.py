@@ -217,32 +217,44 @@ def make_room(cfg, prec, rank, world, local_rank, transport, stream, tb_want):
     return room, tb, t_create, plan
 
 
+GRAPH_WARM = 32  # untimed steps that instantiate the CUDA graphs of both buffer parities
+
+
 def time_room(room, steps, warmup, stream, world, clk=None):
-    """W untimed steps, then K steps between CUDA events on the room's stream
-    (barrier + synchronize on both sides); per-kernel CUDA-event times."""
+    """W untimed warm-up steps (+ GRAPH_WARM more that build the step graphs),
+    then K steps between CUDA events on the room's stream (barrier +
+    synchronize on both sides): the product path, CUDA graphs of 16 steps.
+    Then K more steps launched kernel by kernel with CUDA events around every
+    kernel (profiling mode), for the per-kernel times only."""
+    import contextlib
     room.step(warmup)
+    room.step(GRAPH_WARM)
     room.synchronize()
     room.read_receivers()
-    room.set_profiling(True)
-    n0 = room.launch_count()
-    ev0 = torch.cuda.Event(enable_timing=True)
-    ev1 = torch.cuda.Event(enable_timing=True)
-    if world > 1:
-        torch.distributed.barrier()
-    torch.cuda.synchronize()
-    import contextlib
-    with (clk if clk is not None else contextlib.nullcontext()):
-        with torch.cuda.stream(stream):
-            ev0.record(stream)
-            room.step(steps)
-            ev1.record(stream)
+
+    def timed(profile, sampler):
+        room.set_profiling(profile)
+        n0 = room.launch_count()
+        ev0 = torch.cuda.Event(enable_timing=True)
+        ev1 = torch.cuda.Event(enable_timing=True)
+        if world > 1:
+            torch.distributed.barrier()
         torch.cuda.synchronize()
-    if world > 1:
-        torch.distributed.barrier()
-    ms = ev0.elapsed_time(ev1)
-    launches = room.launch_count() - n0
-    kt = room.get_kernel_times()
-    room.set_profiling(False)
+        with (sampler if sampler is not None else contextlib.nullcontext()):
+            with torch.cuda.stream(stream):
+                ev0.record(stream)
+                room.step(steps)
+                ev1.record(stream)
+            torch.cuda.synchronize()
+        if world > 1:
+            torch.distributed.barrier()
+        kt = room.get_kernel_times() if profile else None
+        room.set_profiling(False)
+        return ev0.elapsed_time(ev1), room.launch_count() - n0, kt
+
+    ms, launches, _ = timed(False, clk)
+    ms_prof, _, kt = timed(True, None)
+    kt["profiled_ms"] = ms_prof
     rec = room.read_receivers()
     return ms, launches, kt, rec
 
@@ -355,7 +367,9 @@ def run_rafd(args, rank, world, local_rank):
                 "halo_transport": args.transport if world > 1 else None,
                 "n_boundary_rank0": info["n_boundary"], "parallelism": f"z-slab x{world}",
                 "l2": "inputs larger than L2 (working set %.1f GB/GPU vs 126 MB L2)" % (info["device_bytes"] / 1e9),
-                "timed": "profiled launches (CUDA events around every kernel) on the room stream",
+                "timed": "CUDA events on the room stream around K steps replayed from CUDA graphs (the product "
+                         "path) after W + %d untimed steps; per-kernel times from K more steps launched with "
+                         "events around every kernel" % GRAPH_WARM,
                 "steps_per_sweep": tb,
                 # RAFD_BENCH_DEVICE pins every rank to one GPU (a functional check of the
                 # multi-rank path): the ranks then share that GPU's bandwidth
@@ -376,6 +390,8 @@ def run_rafd(args, rank, world, local_rank):
             "kernels": {
                 "volume_ms_per_step": round(vol_ms, 5), "boundary_ms_per_step": round(bnd_ms, 5),
                 "other_ms_per_step": round(kt["other_ms"] / args.steps, 5),
+                # the same K steps launched kernel by kernel with events around each
+                "profiled_ms_per_step": round(kt["profiled_ms"] / args.steps, 5),
                 "shell_ms_per_step": round(kt["shell_ms"] / args.steps, 5),
                 "n_shell": info["n_shell"],
                 "boundary_gbs": None if bnd_gbs is None else round(bnd_gbs, 1),

@@ -94,6 +94,10 @@ template <typename T> struct FusedArgs {
     // dynamic unit scheduling (set by the plan): [2] atomic unit counter and
     // CTAs-done count, reset by the last CTA; nullptr = static round-robin
     unsigned int *work;
+    // units that hold an inside voxel (set by the plan for whole-room launches of
+    // non-cuboid rooms): chunk << 16 | tile, ascending; nullptr = every unit
+    const uint32_t *ulist;
+    int nulist;
 };
 
 // plan == nullptr selects the one-thread-per-voxel v0 kernel (A/B reference);
