@@ -67,6 +67,51 @@ def test_c4_full_size_two_steps_bitwise(orc):
         assert np.array_equal(r.read_receivers(), rec_o)
 
 
+def test_c4_full_size_many_steps_bitwise(orc):
+    """The bench configuration over many launches: C4 with temporal blocking,
+    37 steps in one rafd_step call (two 16-step CUDA graphs of double steps,
+    then two double steps and a single step), so the dynamic unit counter of
+    k_volume2 is reset and reused across 18 launches and the graph and direct
+    paths hand the state to each other.  Every voxel, the branch state and
+    the receivers bitwise against the oracle (the oracle runs on all host
+    cores)."""
+    cfg = bench.workload("C4", 1)
+    nx, ny, nz = cfg["room"]
+    beta0, D, E, F = I.config_materials(cfg)
+    dev = torch.device("cuda", 0)
+    mask_d, mm_d, _ = bench.slab_inputs(cfg, 0, nz, dev)
+    g = rafd.Room(mask_d, LAM, 32, beta0, D, E, F, matmap=mm_d)
+    g.set_temporal_blocking(2)
+    gen = torch.Generator(device=dev).manual_seed(37)
+    up = torch.rand((nz, ny, nx), generator=gen, device=dev, dtype=torch.float32) * 2 - 1
+    uc = torch.rand((nz, ny, nx), generator=gen, device=dev, dtype=torch.float32) * 2 - 1
+    src = I.source_position((nx, ny, nz))
+    rcv = I.receiver_positions((nx, ny, nz))
+    sig = I.gaussian_pulse(24, 4.0)
+    g.set_state(up, uc)
+    g.set_source(src, sig)
+    g.set_receivers(rcv)
+    g.step(37)
+    o = orc.OracleRoom(mask_d.cpu().numpy(), LAM, 32, beta0, D, E, F, matmap=mm_d.cpu().numpy())
+    del mask_d, mm_d
+    o.set_state(up.cpu().numpy(), uc.cpu().numpy())
+    del up, uc
+    o.set_source(src, sig)
+    o.set_receivers(rcv)
+    o.step(37)
+    cur_o, prv_o = o.read_field()
+    cur_g = torch.empty((nz, ny, nx), dtype=torch.float32, device=dev)
+    prv_g = torch.empty_like(cur_g)
+    g.read_field(out_curr=cur_g, out_prev=prv_g)
+    assert np.array_equal(cur_g.cpu().numpy(), cur_o)
+    assert np.array_equal(prv_g.cpu().numpy(), prv_o)
+    del cur_g, prv_g
+    vg, gg = g.read_branch_state()
+    vo, go = o.read_branch_state()
+    assert np.array_equal(vg, vo) and np.array_equal(gg, go)
+    assert np.array_equal(g.read_receivers(), o.read_receivers())
+
+
 @pytest.mark.parametrize("name,precision,steps", [("C2a", 32, 30), ("C2b", 32, 30), ("C3", 32, 12), ("C3d", 64, 12)])
 def test_config_full_size_bitwise(orc, name, precision, steps):
     """BASELINE.json configs[1..2] at full size (256^3 L-shape and dome with
