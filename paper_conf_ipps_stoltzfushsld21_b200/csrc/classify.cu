@@ -291,11 +291,22 @@ __global__ void k_compact(Grid g, const uint8_t *__restrict__ K, const int64_t *
     });
 }
 
+// the shell list and, per entry, which of its six face neighbours are inside
+// (bit 0..5: x-1, x+1, y-1, y+1, z-1, z+1; ghost-plane bytes carry the 0x80
+// inside flag): the shell kernel loads only inside neighbours -- an outside
+// voxel holds +0 -- and takes K as the popcount, so it reads no K byte
 template <typename IdxT>
 __global__ void k_shell_compact(Grid g, const uint8_t *__restrict__ K, const int64_t *__restrict__ off,
-                                IdxT *__restrict__ list)
+                                IdxT *__restrict__ list, uint8_t *__restrict__ nmask)
 {
-    rows_compact<kSelShell>(g, K, off, [&](int64_t i, int64_t pos, int64_t, uint8_t) { list[i] = (IdxT)pos; });
+    rows_compact<kSelShell>(g, K, off, [&](int64_t i, int64_t pos, int64_t, uint8_t) {
+        list[i] = (IdxT)pos;
+        const int64_t d[6] = {-1, 1, -g.pitch, g.pitch, -g.plane, g.plane};
+        uint32_t m = 0;
+#pragma unroll
+        for (int k = 0; k < 6; k++) m |= (K[pos + d[k]] != 0) << k;
+        nmask[i] = (uint8_t)m;
+    });
 }
 
 __global__ void k_gather_mat(const uint8_t *__restrict__ mm, int64_t canon0,
@@ -381,12 +392,12 @@ cudaError_t launch_shell_counts(const Grid &g, const uint8_t *K, int64_t *counts
 }
 
 cudaError_t launch_shell_compact(const Grid &g, const uint8_t *K, const int64_t *off, bool idx64, void *list,
-                                 cudaStream_t s)
+                                 uint8_t *nmask, cudaStream_t s)
 {
     const int64_t rows = (int64_t)g.lnz * g.ny;
     if (rows == 0) return cudaSuccess;
-    if (idx64) k_shell_compact<int64_t><<<row_blocks(rows), 256, 0, s>>>(g, K, off, (int64_t *)list);
-    else k_shell_compact<uint32_t><<<row_blocks(rows), 256, 0, s>>>(g, K, off, (uint32_t *)list);
+    if (idx64) k_shell_compact<int64_t><<<row_blocks(rows), 256, 0, s>>>(g, K, off, (int64_t *)list, nmask);
+    else k_shell_compact<uint32_t><<<row_blocks(rows), 256, 0, s>>>(g, K, off, (uint32_t *)list, nmask);
     return cudaGetLastError();
 }
 

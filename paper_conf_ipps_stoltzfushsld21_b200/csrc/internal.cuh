@@ -157,7 +157,7 @@ cudaError_t launch_compact(const Grid &g, const uint8_t *K, const int64_t *row_o
 // with K < 6): per-row counts and the ascending list of padded positions
 cudaError_t launch_shell_counts(const Grid &g, const uint8_t *K, int64_t *counts, cudaStream_t s);
 cudaError_t launch_shell_compact(const Grid &g, const uint8_t *K, const int64_t *off, bool idx64, void *list,
-                                 cudaStream_t s);
+                                 uint8_t *nmask, cudaStream_t s);
 cudaError_t launch_gather_mat(const uint8_t *matmap_chunk, int64_t canon0, const int64_t *bidx,
                               int64_t i_lo, int64_t i_hi, uint8_t *matb, int M,
                               unsigned int *bad_flag, cudaStream_t s);

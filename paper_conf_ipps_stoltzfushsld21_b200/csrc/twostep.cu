@@ -366,7 +366,8 @@ __global__ void __launch_bounds__(TbGeom<T, TY, SU, SP>::NT, 1)
 // is then the sub-range of those planes and star entries elsewhere are skipped
 // (its edge planes are recomputed whole from the exchanged u^{n+1}).
 template <typename T, typename IdxT>
-__global__ void __launch_bounds__(256) k_shell(const IdxT *__restrict__ list, int64_t n, const int64_t *__restrict__ src,
+__global__ void __launch_bounds__(256) k_shell(const IdxT *__restrict__ list, const uint8_t *__restrict__ nmask,
+                                               int64_t n, const int64_t *__restrict__ src,
                                                const T *__restrict__ u1, const T *__restrict__ u0,
                                                const uint8_t *__restrict__ K, T *__restrict__ out, Grid g, T l2,
                                                int zp_lo, int zp_hi)
@@ -377,11 +378,26 @@ __global__ void __launch_bounds__(256) k_shell(const IdxT *__restrict__ list, in
     const int64_t p = i < n ? (int64_t)list[i] : src[i - n];
     if (p < 0) return;
     if (i >= n && (p < (int64_t)zp_lo * g.plane || p >= (int64_t)zp_hi * g.plane)) return;
-    // every load depends only on p: all of them in flight together (one
-    // dependent round trip after the list entry instead of two)
-    const int nbr = K[p];
-    const T xm = u1[p - 1], xp = u1[p + 1], ym = u1[p - g.pitch], yp = u1[p + g.pitch];
-    const T zm = u1[p - g.plane], zp = u1[p + g.plane], c = u1[p], pv = u0[p];
+    // which face neighbours are inside: list entries carry it (no K load);
+    // the source's star entries read K.  An outside neighbour holds +0, so it
+    // is not loaded.  Every load depends only on p and the mask: all of them in
+    // flight together.
+    uint32_t m;
+    int nbr;
+    if (i < n) {
+        m = nmask[i];
+        nbr = __popc(m);
+    } else {
+        const int64_t d[6] = {-1, 1, -g.pitch, g.pitch, -g.plane, g.plane};
+        m = 0;
+#pragma unroll
+        for (int k = 0; k < 6; k++) m |= (K[p + d[k]] != 0) << k;
+        nbr = K[p];
+    }
+    const T xm = (m & 1) ? u1[p - 1] : (T)0, xp = (m & 2) ? u1[p + 1] : (T)0;
+    const T ym = (m & 4) ? u1[p - g.pitch] : (T)0, yp = (m & 8) ? u1[p + g.pitch] : (T)0;
+    const T zm = (m & 16) ? u1[p - g.plane] : (T)0, zp = (m & 32) ? u1[p + g.plane] : (T)0;
+    const T c = u1[p], pv = u0[p];
     T s = R::add(xm, xp);
     s = R::add(s, ym);
     s = R::add(s, yp);
@@ -391,8 +407,7 @@ __global__ void __launch_bounds__(256) k_shell(const IdxT *__restrict__ list, in
     T t = R::mul(a, c);
     t = R::add(t, R::mul(l2, s));
     // an outside voxel (a star entry with K = 0) holds +0 in every buffer, so
-    // storing u0 there changes nothing -- and the store then needs every load
-    // (the compiler cannot sink any of them below a K test)
+    // storing u0 there changes nothing
     out[p] = nbr != 0 ? R::sub(t, pv) : pv;
 }
 
@@ -429,6 +444,7 @@ struct TwoStepPlan {
     CUtensorMap umap[4], pmap[4], kmap;
     int tiles_x, tiles_y, grid, smem;
     void *list = nullptr;  // shell positions (uint32 or int64), ascending
+    uint8_t *nmask = nullptr;  // per shell entry: inside face neighbours (bits x-1, x+1, y-1, y+1, z-1, z+1)
     int64_t n_shell = 0;
     int64_t sh_lo = 0, sh_hi = 0;  // list range of the local planes [1, lnz-1) (slab interior)
     int64_t *src = nullptr;  // [7] the source's star, -1 = none
@@ -501,7 +517,8 @@ cudaError_t twostep_plan_create(const Grid &g, void *const u[4], uint8_t *K_allo
         e = cudaMemcpyAsync(&pl->sh_hi, off + (int64_t)(g.lnz - 1) * g.ny, 8, cudaMemcpyDeviceToHost, s);
     if (e == cudaSuccess) e = cudaStreamSynchronize(s);
     if (e == cudaSuccess) e = dev_alloc((void **)&pl->list, (size_t)std::max<int64_t>(n, 1) * (idx64 ? 8 : 4));
-    if (e == cudaSuccess && n > 0) e = launch_shell_compact(g, K, off, idx64, pl->list, s);
+    if (e == cudaSuccess) e = dev_alloc((void **)&pl->nmask, (size_t)std::max<int64_t>(n, 1));
+    if (e == cudaSuccess && n > 0) e = launch_shell_compact(g, K, off, idx64, pl->list, pl->nmask, s);
     if (e == cudaSuccess) e = dev_alloc((void **)&pl->work, 2 * sizeof(unsigned int));
     if (e == cudaSuccess) e = cudaMemsetAsync(pl->work, 0, 2 * sizeof(unsigned int), s);
     if (e == cudaSuccess) e = dev_alloc((void **)&pl->src, 7 * 8);
@@ -513,6 +530,7 @@ cudaError_t twostep_plan_create(const Grid &g, void *const u[4], uint8_t *K_allo
     pl->n_shell = n;
     if (e != cudaSuccess) {
         if (pl->list) dev_free(pl->list);
+        if (pl->nmask) dev_free(pl->nmask);
         if (pl->src) dev_free(pl->src);
         if (pl->work) dev_free(pl->work);
         delete pl;
@@ -528,6 +546,7 @@ void twostep_plan_destroy(void *plan)
     auto *pl = (TwoStepPlan *)plan;
     if (!pl) return;
     if (pl->list) dev_free(pl->list);
+    if (pl->nmask) dev_free(pl->nmask);
     if (pl->src) dev_free(pl->src);
     if (pl->work) dev_free(pl->work);
     delete pl;
@@ -616,10 +635,10 @@ cudaError_t launch_shell(const void *plan, const Grid &g, const T *u1, const T *
     const int64_t n = cnt + 7;
     const unsigned blocks = (unsigned)((n + 255) / 256);
     if (pl->idx64)
-        k_shell<T, int64_t><<<blocks, 256, 0, s>>>((const int64_t *)pl->list + lo, cnt, pl->src, u1, u0, K, out, g,
+        k_shell<T, int64_t><<<blocks, 256, 0, s>>>((const int64_t *)pl->list + lo, pl->nmask + lo, cnt, pl->src, u1, u0, K, out, g,
                                                    l2, zp_lo, zp_hi);
     else
-        k_shell<T, uint32_t><<<blocks, 256, 0, s>>>((const uint32_t *)pl->list + lo, cnt, pl->src, u1, u0, K, out, g,
+        k_shell<T, uint32_t><<<blocks, 256, 0, s>>>((const uint32_t *)pl->list + lo, pl->nmask + lo, cnt, pl->src, u1, u0, K, out, g,
                                                     l2, zp_lo, zp_hi);
     return cudaGetLastError();
 }
