@@ -131,6 +131,14 @@ cudaError_t launch_volume2(const void *plan, const Grid &g, int cur_buf, int pre
 template <typename T>
 cudaError_t launch_shell(const void *plan, const Grid &g, const T *u1, const T *u0, const uint8_t *K, T *out,
                          double lambda, cudaStream_t s, bool interior = false);
+// the shell fused with the step-(n+2) boundary update and the source /
+// receivers (whole rooms; the list's node entries must be exactly the room's
+// nodes: twostep_shell_nodes(plan) == Nb)
+template <typename T>
+cudaError_t launch_shell_bnd(const void *plan, const Grid &g, const T *u1, const T *u0, const uint8_t *K, T *out,
+                             double lambda, int MB, const uint8_t *matb, T *ub, T *gst, T *vst, int64_t Nb,
+                             const T *tab, int M, Ctl<T> *ctl, unsigned int *ticket, cudaStream_t s);
+int64_t twostep_shell_nodes(const void *plan);
 template <typename T>
 cudaError_t launch_boundary(int MB, bool idx64, const void *bpos, const uint8_t *Kb,
                             const uint8_t *matb, int64_t i_lo, int64_t i_hi, int64_t Nb, T *unext,

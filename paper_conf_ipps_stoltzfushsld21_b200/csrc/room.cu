@@ -131,6 +131,7 @@ struct rafd_room {
     void *tab = nullptr;   // T: beta[M] | BI | D | DI | F  ([M*MB] each)
     std::vector<unsigned char> tab_host;  // the same table on the host (boundary-kernel launch parameter)
     bool use_pool = false;                // buffers through the library's memory cache (whole rooms)
+    bool shell_bnd = false;               // double steps fuse the shell with the step-(n+2) boundary pass
     double *DF = nullptr;  // double D | F for the energy hook
     void *ctl = nullptr;   // Ctl<T>
     unsigned int *ticket = nullptr;  // last-block ticket of the boundary kernel's fused source/receivers
@@ -827,6 +828,14 @@ template <typename T> static cudaError_t enqueue_step2(rafd_room *r, int pair, i
     };
     cudaError_t e = timed_launch(r, s, prof, 0, [&] { return launch_volume2<T>(r->tbplan, g, bB, bA, C, D, r->lambda, s); });
     if (e == cudaSuccess) e = bnd_src(C, cur);
+    if (e == cudaSuccess && r->shell_bnd) {
+        // the shell, the step-(n+2) boundary update and the source / receivers in one pass
+        return timed_launch(r, s, prof, 3, [&] {
+            return launch_shell_bnd<T>(r->tbplan, g, C, B, r->K, D, r->lambda, r->MB, r->matb, ub_slot<T>(r, cur ^ 1),
+                                       (T *)r->gst, (T *)r->vst, r->nb, (const T *)r->tab, r->M, ctl_of<T>(r),
+                                       r->ticket, s);
+        });
+    }
     if (e == cudaSuccess)
         e = timed_launch(r, s, prof, 3, [&] { return launch_shell<T>(r->tbplan, g, C, B, r->K, D, r->lambda, s); });
     if (e == cudaSuccess) e = bnd_src(D, cur ^ 1);
@@ -1061,7 +1070,9 @@ static cudaError_t slab_step(rafd_room *r, bool two, bool prof, int64_t n)
 // (whole room: the boundary kernel runs the source/receivers in its last block;
 // fused / single-kernel schemes and rooms without boundary nodes launch k_src_rcv)
 static int kernels_per_step(const rafd_room *) { return 2; }
-static int kernels_per_double_step(const rafd_room *) { return 4; }
+// k_volume2, the step-(n+1) boundary kernel, and the shell + step-(n+2)
+// boundary (fused: one kernel; else two)
+static int kernels_per_double_step(const rafd_room *r) { return r->shell_bnd ? 3 : 4; }
 
 // a graph of G steps from the state (pair, cur) (index pair + cur); it ends in
 // the same state (G single steps flip cur an even number of times, G/2 double
@@ -1672,6 +1683,13 @@ template <typename T> static int enable_twostep_t(rafd_room *r)
     r->vplan = vp;
     r->tbplan = tp;
     r->n_shell = nsh;
+    // the fused shell + boundary pass needs the list's node entries to be the
+    // room's nodes (always, for a whole room); RAFD_SHELL_BND=0 keeps two passes
+    {
+        const char *sb = getenv("RAFD_SHELL_BND");
+        r->shell_bnd = r->nranks == 1 && r->nb > 0 && r->scheme == 0 && twostep_shell_nodes(tp) == r->nb &&
+                       !(sb && strcmp(sb, "0") == 0);
+    }
     r->device_bytes += r->n_shell * (r->idx64 ? 8 : 4) + 56;
     for (int k = 2; k < 4; k++) r->u[k] = nu[k];
     return RAFD_OK;

@@ -32,6 +32,7 @@
 
 #include <stdlib.h>
 
+#include "bnd_math.cuh"
 #include "internal.cuh"
 
 namespace rafd {
@@ -411,6 +412,114 @@ __global__ void __launch_bounds__(256) k_shell(const IdxT *__restrict__ list, co
     out[p] = nbr != 0 ? R::sub(t, pv) : pv;
 }
 
+// ---- the shell fused with the step-(n+2) boundary update (whole rooms).
+// Every boundary node is a shell voxel, and the shell list and the node list
+// are both in ascending position order, so the k-th node entry of the shell
+// list is node k: its index is the node count of the entry's 32-entry group
+// (wbase, built with the plan) plus the nodes before it in its warp (ballot).
+// Per entry: the volume value of step n+2 from the final u^{n+1} (as k_shell),
+// then, at a node, Listing 3/4's update of it with the node's state (as
+// k_boundary, DESIGN.md §4 order), one store of the final value.  The last
+// block adds the source and records the receivers (as k_boundary).  The
+// source's star entries that are shell voxels are left to their list entry.
+template <typename T, int MB, typename IdxT>
+__global__ void __launch_bounds__(256)
+    k_shell_bnd(const IdxT *__restrict__ list, const uint8_t *__restrict__ nmask, const int64_t *__restrict__ wbase,
+                int64_t n, const int64_t *__restrict__ src, const T *__restrict__ u1, const T *__restrict__ u0,
+                const uint8_t *__restrict__ K, T *__restrict__ out, Grid g, T l2, T l,
+                const uint8_t *__restrict__ matb, T *__restrict__ ub, T *__restrict__ gst, T *__restrict__ vst,
+                int64_t Nb, const T *__restrict__ tab, int M, Ctl<T> *ctl, unsigned int *ticket)
+{
+    using R = rn<T>;
+    const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    const int lane = threadIdx.x & 31;
+    const bool in_list = i < n;
+    int64_t p = -1;
+    uint32_t m = 0;
+    int nbr = 0;
+    if (in_list) {
+        p = (int64_t)list[i];
+        m = nmask[i];
+        nbr = __popc(m);
+    } else if (i < n + 7) {
+        p = src[i - n];
+        if (p >= 0) {  // a star voxel: recomputed here unless it is a shell voxel (its list entry does it)
+            const int64_t d[6] = {-1, 1, -g.pitch, g.pitch, -g.plane, g.plane};
+            nbr = K[p];
+            bool shell = nbr < 6;
+#pragma unroll
+            for (int k = 0; k < 6; k++) {
+                const int kn = K[p + d[k]];
+                m |= (kn != 0) << k;
+                shell = shell || kn < 6;
+            }
+            if (nbr == 0 || shell) p = -1;
+        }
+    }
+    const bool node = in_list && nbr < 6;
+    const unsigned bal = __ballot_sync(0xffffffffu, node);
+    const int64_t rank = node ? wbase[i >> 5] + __popc(bal & ((1u << lane) - 1u)) : 0;
+    if (p >= 0) {
+        T uprev = (T)0, gb[MB > 0 ? MB : 1], vb[MB > 0 ? MB : 1];
+        int mi = 0;
+        if (node) {  // issued with the stencil loads
+            mi = matb[rank];
+            uprev = ub[rank];
+#pragma unroll
+            for (int b = 0; b < MB; b++) {
+                gb[b] = gst[(int64_t)b * Nb + rank];
+                vb[b] = vst[(int64_t)b * Nb + rank];
+            }
+        }
+        const T xm = (m & 1) ? u1[p - 1] : (T)0, xp = (m & 2) ? u1[p + 1] : (T)0;
+        const T ym = (m & 4) ? u1[p - g.pitch] : (T)0, yp = (m & 8) ? u1[p + g.pitch] : (T)0;
+        const T zm = (m & 16) ? u1[p - g.plane] : (T)0, zp = (m & 32) ? u1[p + g.plane] : (T)0;
+        const T c = u1[p], pv = u0[p];
+        T s = R::add(xm, xp);
+        s = R::add(s, ym);
+        s = R::add(s, yp);
+        s = R::add(s, zm);
+        s = R::add(s, zp);
+        const T a = R::sub((T)2, R::mul(l2, (T)nbr));
+        T t = R::mul(a, c);
+        t = R::add(t, R::mul(l2, s));
+        T x = R::sub(t, pv);
+        if (node) {
+            x = bnd_math<T, MB>(x, uprev, nbr, mi, tab, M, l, gb, vb);
+#pragma unroll
+            for (int b = 0; b < MB; b++) {
+                gst[(int64_t)b * Nb + rank] = gb[b];
+                vst[(int64_t)b * Nb + rank] = vb[b];
+            }
+            ub[rank] = x;  // u^{n+2} at the node: read back as u^n two steps later
+        }
+        out[p] = x;
+    }
+    // the last block adds the source and records the receivers
+    __shared__ int last;
+    __shared__ __align__(16) Ctl<T> cb;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        __threadfence();
+        last = atomicAdd(ticket, 1u) == gridDim.x - 1;
+    }
+    __syncthreads();
+    if (last) {
+        __threadfence();
+        src_rcv_block<T>(out, ub, ctl, 3, 0, 0, cb);
+        if (threadIdx.x == 0) *ticket = 0u;
+    }
+}
+
+// node count of every 32-entry group of the shell list
+__global__ void k_shell_wcount(const uint8_t *__restrict__ nmask, int64_t n, int64_t *__restrict__ cnt)
+{
+    const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    const bool node = i < n && __popc(nmask[i]) < 6;
+    const unsigned b = __ballot_sync(0xffffffffu, node);
+    if ((threadIdx.x & 31) == 0 && i < n) cnt[i >> 5] = __popc(b);
+}
+
 // ------------------------------------------------------------------ host side
 static PFN_cuTensorMapEncodeTiled_v12000 tb_encode_fn()
 {
@@ -445,6 +554,8 @@ struct TwoStepPlan {
     int tiles_x, tiles_y, grid, smem;
     void *list = nullptr;  // shell positions (uint32 or int64), ascending
     uint8_t *nmask = nullptr;  // per shell entry: inside face neighbours (bits x-1, x+1, y-1, y+1, z-1, z+1)
+    int64_t *wbase = nullptr;  // [n/32 + 1] boundary nodes before each 32-entry group of the list
+    int64_t n_nodes = 0;       // boundary nodes in the list
     int64_t n_shell = 0;
     int64_t sh_lo = 0, sh_hi = 0;  // list range of the local planes [1, lnz-1) (slab interior)
     int64_t *src = nullptr;  // [7] the source's star, -1 = none
@@ -519,6 +630,25 @@ cudaError_t twostep_plan_create(const Grid &g, void *const u[4], uint8_t *K_allo
     if (e == cudaSuccess) e = dev_alloc((void **)&pl->list, (size_t)std::max<int64_t>(n, 1) * (idx64 ? 8 : 4));
     if (e == cudaSuccess) e = dev_alloc((void **)&pl->nmask, (size_t)std::max<int64_t>(n, 1));
     if (e == cudaSuccess && n > 0) e = launch_shell_compact(g, K, off, idx64, pl->list, pl->nmask, s);
+    // node count per 32-entry group, scanned (the fused shell + boundary kernel)
+    const int64_t ngr = (n + 31) / 32;
+    int64_t *wcnt = nullptr;
+    void *wtmp = nullptr;
+    size_t wtb = 0;
+    if (e == cudaSuccess) e = dev_alloc((void **)&wcnt, (size_t)(ngr + 1) * 8);
+    if (e == cudaSuccess) e = dev_alloc((void **)&pl->wbase, (size_t)(ngr + 1) * 8);
+    if (e == cudaSuccess) e = cudaMemsetAsync(wcnt, 0, (size_t)(ngr + 1) * 8, s);
+    if (e == cudaSuccess && n > 0) {
+        k_shell_wcount<<<(unsigned)((n + 255) / 256), 256, 0, s>>>(pl->nmask, n, wcnt);
+        e = cudaGetLastError();
+    }
+    if (e == cudaSuccess) e = exclusive_scan_rows64(wcnt, pl->wbase, ngr + 1, nullptr, &wtb, s);
+    if (e == cudaSuccess) e = dev_alloc(&wtmp, wtb ? wtb : 16);
+    if (e == cudaSuccess) e = exclusive_scan_rows64(wcnt, pl->wbase, ngr + 1, wtmp, &wtb, s);
+    if (e == cudaSuccess) e = cudaMemcpyAsync(&pl->n_nodes, pl->wbase + ngr, 8, cudaMemcpyDeviceToHost, s);
+    if (e == cudaSuccess) e = cudaStreamSynchronize(s);
+    if (wcnt) dev_free(wcnt);
+    if (wtmp) dev_free(wtmp);
     if (e == cudaSuccess) e = dev_alloc((void **)&pl->work, 2 * sizeof(unsigned int));
     if (e == cudaSuccess) e = cudaMemsetAsync(pl->work, 0, 2 * sizeof(unsigned int), s);
     if (e == cudaSuccess) e = dev_alloc((void **)&pl->src, 7 * 8);
@@ -531,6 +661,7 @@ cudaError_t twostep_plan_create(const Grid &g, void *const u[4], uint8_t *K_allo
     if (e != cudaSuccess) {
         if (pl->list) dev_free(pl->list);
         if (pl->nmask) dev_free(pl->nmask);
+        if (pl->wbase) dev_free(pl->wbase);
         if (pl->src) dev_free(pl->src);
         if (pl->work) dev_free(pl->work);
         delete pl;
@@ -547,10 +678,13 @@ void twostep_plan_destroy(void *plan)
     if (!pl) return;
     if (pl->list) dev_free(pl->list);
     if (pl->nmask) dev_free(pl->nmask);
+    if (pl->wbase) dev_free(pl->wbase);
     if (pl->src) dev_free(pl->src);
     if (pl->work) dev_free(pl->work);
     delete pl;
 }
+
+int64_t twostep_shell_nodes(const void *plan) { return plan ? ((const TwoStepPlan *)plan)->n_nodes : -1; }
 
 cudaError_t twostep_set_source(void *plan, int64_t pos, const Grid &g)
 {
@@ -643,13 +777,58 @@ cudaError_t launch_shell(const void *plan, const Grid &g, const T *u1, const T *
     return cudaGetLastError();
 }
 
+template <typename T, int MB>
+static cudaError_t launch_sb(const TwoStepPlan *pl, const Grid &g, const T *u1, const T *u0, const uint8_t *K,
+                             T *out, T l2, T l, const uint8_t *matb, T *ub, T *gst, T *vst, int64_t Nb, const T *tab,
+                             int M, Ctl<T> *ctl, unsigned int *ticket, cudaStream_t s)
+{
+    const int64_t n = pl->n_shell;
+    const unsigned blocks = (unsigned)((n + 7 + 255) / 256);
+    if (pl->idx64)
+        k_shell_bnd<T, MB, int64_t><<<blocks, 256, 0, s>>>((const int64_t *)pl->list, pl->nmask, pl->wbase, n, pl->src,
+                                                           u1, u0, K, out, g, l2, l, matb, ub, gst, vst, Nb, tab, M,
+                                                           ctl, ticket);
+    else
+        k_shell_bnd<T, MB, uint32_t><<<blocks, 256, 0, s>>>((const uint32_t *)pl->list, pl->nmask, pl->wbase, n,
+                                                            pl->src, u1, u0, K, out, g, l2, l, matb, ub, gst, vst, Nb,
+                                                            tab, M, ctl, ticket);
+    return cudaGetLastError();
+}
+
+template <typename T>
+cudaError_t launch_shell_bnd(const void *plan, const Grid &g, const T *u1, const T *u0, const uint8_t *K, T *out,
+                             double lambda, int MB, const uint8_t *matb, T *ub, T *gst, T *vst, int64_t Nb,
+                             const T *tab, int M, Ctl<T> *ctl, unsigned int *ticket, cudaStream_t s)
+{
+    const auto *pl = (const TwoStepPlan *)plan;
+    const T l2 = (T)(lambda * lambda), l = (T)lambda;
+#define RAFD_SB(k) \
+    case k: return launch_sb<T, k>(pl, g, u1, u0, K, out, l2, l, matb, ub, gst, vst, Nb, tab, M, ctl, ticket, s);
+    switch (MB) {
+        RAFD_SB(0)
+        RAFD_SB(1)
+        RAFD_SB(2)
+        RAFD_SB(3)
+        RAFD_SB(4)
+        RAFD_SB(5)
+        RAFD_SB(6)
+        RAFD_SB(7)
+        RAFD_SB(8)
+        default: return cudaErrorInvalidValue;
+    }
+#undef RAFD_SB
+}
+
 #define RAFD_TB_INST(T)                                                                                            \
     template cudaError_t twostep_plan_create<T>(const Grid &, void *const[4], uint8_t *, const uint8_t *, bool, int, \
                                                 cudaStream_t, void **, int64_t *);                                  \
     template cudaError_t launch_volume2<T>(const void *, const Grid &, int, int, T *, T *, double, cudaStream_t,    \
                                            int, int);                                                               \
     template cudaError_t launch_shell<T>(const void *, const Grid &, const T *, const T *, const uint8_t *, T *,     \
-                                         double, cudaStream_t, bool);
+                                         double, cudaStream_t, bool);                                                 \
+    template cudaError_t launch_shell_bnd<T>(const void *, const Grid &, const T *, const T *, const uint8_t *, T *, \
+                                             double, int, const uint8_t *, T *, T *, T *, int64_t, const T *, int,   \
+                                             Ctl<T> *, unsigned int *, cudaStream_t);
 RAFD_TB_INST(float)
 RAFD_TB_INST(double)
 #undef RAFD_TB_INST
