@@ -422,7 +422,7 @@ __global__ void __launch_bounds__(256) k_shell(const IdxT *__restrict__ list, co
 // k_boundary, DESIGN.md §4 order), one store of the final value.  The last
 // block adds the source and records the receivers (as k_boundary).  The
 // source's star entries that are shell voxels are left to their list entry.
-template <typename T, int MB, typename IdxT>
+template <typename T, int MB, typename IdxT, int ENT>
 __global__ void __launch_bounds__(256)
     k_shell_bnd(const IdxT *__restrict__ list, const uint8_t *__restrict__ nmask, const int64_t *__restrict__ wbase,
                 int64_t n, const int64_t *__restrict__ src, const T *__restrict__ u1, const T *__restrict__ u0,
@@ -431,69 +431,75 @@ __global__ void __launch_bounds__(256)
                 int64_t Nb, const T *__restrict__ tab, int M, Ctl<T> *ctl, unsigned int *ticket)
 {
     using R = rn<T>;
-    const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     const int lane = threadIdx.x & 31;
-    const bool in_list = i < n;
-    int64_t p = -1;
-    uint32_t m = 0;
-    int nbr = 0;
-    if (in_list) {
-        p = (int64_t)list[i];
-        m = nmask[i];
-        nbr = __popc(m);
-    } else if (i < n + 7) {
-        p = src[i - n];
-        if (p >= 0) {  // a star voxel: recomputed here unless it is a shell voxel (its list entry does it)
-            const int64_t d[6] = {-1, 1, -g.pitch, g.pitch, -g.plane, g.plane};
-            nbr = K[p];
-            bool shell = nbr < 6;
+    // ENT entries per thread (entry = block * 256 * ENT + e * 256 + tid): each
+    // warp still covers 32 consecutive entries per e, and the block's ticket
+    // below is paid once per 256 * ENT entries
 #pragma unroll
-            for (int k = 0; k < 6; k++) {
-                const int kn = K[p + d[k]];
-                m |= (kn != 0) << k;
-                shell = shell || kn < 6;
-            }
-            if (nbr == 0 || shell) p = -1;
-        }
-    }
-    const bool node = in_list && nbr < 6;
-    const unsigned bal = __ballot_sync(0xffffffffu, node);
-    const int64_t rank = node ? wbase[i >> 5] + __popc(bal & ((1u << lane) - 1u)) : 0;
-    if (p >= 0) {
-        T uprev = (T)0, gb[MB > 0 ? MB : 1], vb[MB > 0 ? MB : 1];
-        int mi = 0;
-        if (node) {  // issued with the stencil loads
-            mi = matb[rank];
-            uprev = ub[rank];
+    for (int e = 0; e < ENT; e++) {
+        const int64_t i = (int64_t)blockIdx.x * (256 * ENT) + e * 256 + threadIdx.x;
+        const bool in_list = i < n;
+        int64_t p = -1;
+        uint32_t m = 0;
+        int nbr = 0;
+        if (in_list) {
+            p = (int64_t)list[i];
+            m = nmask[i];
+            nbr = __popc(m);
+        } else if (i < n + 7) {
+            p = src[i - n];
+            if (p >= 0) {  // a star voxel: recomputed here unless it is a shell voxel (its list entry does it)
+                const int64_t d[6] = {-1, 1, -g.pitch, g.pitch, -g.plane, g.plane};
+                nbr = K[p];
+                bool shell = nbr < 6;
 #pragma unroll
-            for (int b = 0; b < MB; b++) {
-                gb[b] = gst[(int64_t)b * Nb + rank];
-                vb[b] = vst[(int64_t)b * Nb + rank];
+                for (int k = 0; k < 6; k++) {
+                    const int kn = K[p + d[k]];
+                    m |= (kn != 0) << k;
+                    shell = shell || kn < 6;
+                }
+                if (nbr == 0 || shell) p = -1;
             }
         }
-        const T xm = (m & 1) ? u1[p - 1] : (T)0, xp = (m & 2) ? u1[p + 1] : (T)0;
-        const T ym = (m & 4) ? u1[p - g.pitch] : (T)0, yp = (m & 8) ? u1[p + g.pitch] : (T)0;
-        const T zm = (m & 16) ? u1[p - g.plane] : (T)0, zp = (m & 32) ? u1[p + g.plane] : (T)0;
-        const T c = u1[p], pv = u0[p];
-        T s = R::add(xm, xp);
-        s = R::add(s, ym);
-        s = R::add(s, yp);
-        s = R::add(s, zm);
-        s = R::add(s, zp);
-        const T a = R::sub((T)2, R::mul(l2, (T)nbr));
-        T t = R::mul(a, c);
-        t = R::add(t, R::mul(l2, s));
-        T x = R::sub(t, pv);
-        if (node) {
-            x = bnd_math<T, MB>(x, uprev, nbr, mi, tab, M, l, gb, vb);
+        const bool node = in_list && nbr < 6;
+        const unsigned bal = __ballot_sync(0xffffffffu, node);
+        const int64_t rank = node ? wbase[i >> 5] + __popc(bal & ((1u << lane) - 1u)) : 0;
+        if (p >= 0) {
+            T uprev = (T)0, gb[MB > 0 ? MB : 1], vb[MB > 0 ? MB : 1];
+            int mi = 0;
+            if (node) {  // issued with the stencil loads
+                mi = matb[rank];
+                uprev = ub[rank];
 #pragma unroll
-            for (int b = 0; b < MB; b++) {
-                gst[(int64_t)b * Nb + rank] = gb[b];
-                vst[(int64_t)b * Nb + rank] = vb[b];
+                for (int b = 0; b < MB; b++) {
+                    gb[b] = gst[(int64_t)b * Nb + rank];
+                    vb[b] = vst[(int64_t)b * Nb + rank];
+                }
             }
-            ub[rank] = x;  // u^{n+2} at the node: read back as u^n two steps later
+            const T xm = (m & 1) ? u1[p - 1] : (T)0, xp = (m & 2) ? u1[p + 1] : (T)0;
+            const T ym = (m & 4) ? u1[p - g.pitch] : (T)0, yp = (m & 8) ? u1[p + g.pitch] : (T)0;
+            const T zm = (m & 16) ? u1[p - g.plane] : (T)0, zp = (m & 32) ? u1[p + g.plane] : (T)0;
+            const T c = u1[p], pv = u0[p];
+            T s = R::add(xm, xp);
+            s = R::add(s, ym);
+            s = R::add(s, yp);
+            s = R::add(s, zm);
+            s = R::add(s, zp);
+            const T a = R::sub((T)2, R::mul(l2, (T)nbr));
+            T t = R::mul(a, c);
+            t = R::add(t, R::mul(l2, s));
+            T x = R::sub(t, pv);
+            if (node) {
+                x = bnd_math<T, MB>(x, uprev, nbr, mi, tab, M, l, gb, vb);
+#pragma unroll
+                for (int b = 0; b < MB; b++) {
+                    gst[(int64_t)b * Nb + rank] = gb[b];
+                    vst[(int64_t)b * Nb + rank] = vb[b];
+                }
+                ub[rank] = x;  // u^{n+2} at the node: read back as u^n two steps later
+            }
+            out[p] = x;
         }
-        out[p] = x;
     }
     // the last block adds the source and records the receivers
     __shared__ int last;
@@ -777,19 +783,22 @@ cudaError_t launch_shell(const void *plan, const Grid &g, const T *u1, const T *
     return cudaGetLastError();
 }
 
+static constexpr int kShellEnt = 1;  // entries per thread of k_shell_bnd
+
 template <typename T, int MB>
 static cudaError_t launch_sb(const TwoStepPlan *pl, const Grid &g, const T *u1, const T *u0, const uint8_t *K,
                              T *out, T l2, T l, const uint8_t *matb, T *ub, T *gst, T *vst, int64_t Nb, const T *tab,
                              int M, Ctl<T> *ctl, unsigned int *ticket, cudaStream_t s)
 {
     const int64_t n = pl->n_shell;
-    const unsigned blocks = (unsigned)((n + 7 + 255) / 256);
+    constexpr int ENT = kShellEnt;
+    const unsigned blocks = (unsigned)((n + 7 + 256 * ENT - 1) / (256 * ENT));
     if (pl->idx64)
-        k_shell_bnd<T, MB, int64_t><<<blocks, 256, 0, s>>>((const int64_t *)pl->list, pl->nmask, pl->wbase, n, pl->src,
+        k_shell_bnd<T, MB, int64_t, ENT><<<blocks, 256, 0, s>>>((const int64_t *)pl->list, pl->nmask, pl->wbase, n, pl->src,
                                                            u1, u0, K, out, g, l2, l, matb, ub, gst, vst, Nb, tab, M,
                                                            ctl, ticket);
     else
-        k_shell_bnd<T, MB, uint32_t><<<blocks, 256, 0, s>>>((const uint32_t *)pl->list, pl->nmask, pl->wbase, n,
+        k_shell_bnd<T, MB, uint32_t, ENT><<<blocks, 256, 0, s>>>((const uint32_t *)pl->list, pl->nmask, pl->wbase, n,
                                                             pl->src, u1, u0, K, out, g, l2, l, matb, ub, gst, vst, Nb,
                                                             tab, M, ctl, ticket);
     return cudaGetLastError();
