@@ -28,6 +28,11 @@
  * coefficients BI, DI, beta are derived from the physical (D, E, F, beta0)
  * in double (reading R5) and rounded once to T.
  *
+ * The same oracle is also built with orc_abi.c into librafd_oracle.so, which
+ * exports the product's C-ABI names (rafd_create, rafd_step, ...) with the same
+ * semantics for whole rooms; tests/test_oracle_abi.py drives
+ * it through the product's own Python binding.
+ *
  * Pins: see tests/test_oracle_*.py.  Every function below is pinned there
  * against something other than itself (closed forms, Table II counts,
  * energy invariants, brute-force dense matrices, exact reflection
@@ -86,6 +91,8 @@ int  orc_set_receivers(orc_room *r, int32_t n, const int32_t *xyz);
  * outside voxels are forced to +0.  v, g: T-typed [MB][Nb] (NULL => keep). */
 int  orc_set_state(orc_room *r, const void *u_prev, const void *u_curr, const void *v, const void *g);
 int  orc_step(orc_room *r, int64_t nsteps);
+/* Checkpoint / resume: the step counter indexes the source signal. */
+int  orc_set_step(orc_room *r, int64_t n);
 /* Single-kernel schemes of the paper: 0 = Listings 2-4 (default),
  * 1 = Listing 1 (n_materials = 1, MB = 0, beta = beta0[0]),
  * 2 = Listing 6 naive FI (constants loss1, loss2, reading R17). */

@@ -15,19 +15,23 @@ import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
 _LIB_PATH = os.path.join(_HERE, "liborc.so")
-_SOURCES = ["orc.c", "orc_step.inc", "orc.h"]
+# the same oracle behind the product's C-ABI names (orc_abi.c)
+ABI_LIB_PATH = os.path.join(_HERE, "librafd_oracle.so")
+_SOURCES = ["orc.c", "orc_step.inc", "orc.h", "orc_abi.c"]
 
 CFLAGS = ["-std=c11", "-O2", "-ffp-contract=off", "-fopenmp", "-fPIC", "-shared", "-Wall", "-Wextra",
           "-Wno-unused-parameter"]
 
 
 def build(force: bool = False) -> str:
-    """Compile liborc.so with gcc (no FMA contraction, no fast-math)."""
+    """Compile liborc.so (and librafd_oracle.so, the same oracle under the
+    product's C-ABI names) with gcc (no FMA contraction, no fast-math)."""
     src_m = max(os.path.getmtime(os.path.join(_HERE, s)) for s in _SOURCES)
-    if force or not os.path.exists(_LIB_PATH) or os.path.getmtime(_LIB_PATH) < src_m:
-        tmp = _LIB_PATH + f".tmp{os.getpid()}"
-        subprocess.check_call(["gcc", *CFLAGS, "-o", tmp, os.path.join(_HERE, "orc.c"), "-lm"])
-        os.replace(tmp, _LIB_PATH)
+    for path, srcs in ((_LIB_PATH, ["orc.c"]), (ABI_LIB_PATH, ["orc.c", "orc_abi.c"])):
+        if force or not os.path.exists(path) or os.path.getmtime(path) < src_m:
+            tmp = path + f".tmp{os.getpid()}"
+            subprocess.check_call(["gcc", *CFLAGS, "-o", tmp, *[os.path.join(_HERE, f) for f in srcs], "-lm"])
+            os.replace(tmp, path)
     return _LIB_PATH
 
 
@@ -62,6 +66,7 @@ def lib():
         L.orc_set_receivers.argtypes = [P, C.c_int32, P]
         L.orc_set_state.argtypes = [P, P, P, P, P]
         L.orc_step.argtypes = [P, C.c_int64]
+        L.orc_set_step.argtypes = [P, C.c_int64]
         L.orc_set_scheme.argtypes = [P, C.c_int32, C.c_double, C.c_double]
         L.orc_read_receivers.argtypes = [P, P, C.c_int64, C.POINTER(C.c_int64)]
         L.orc_read_field.argtypes = [P, P, P]
