@@ -253,7 +253,12 @@ def time_room(room, steps, warmup, stream, world, clk=None):
         return ev0.elapsed_time(ev1), room.launch_count() - n0, kt
 
     ms, launches, _ = timed(False, clk)
+    # per-kernel times: the faster of two profiled passes (a single pass is
+    # exposed to one-off slowdowns of a few launches)
     ms_prof, _, kt = timed(True, None)
+    ms_prof2, _, kt2 = timed(True, None)
+    if ms_prof2 < ms_prof:
+        ms_prof, kt = ms_prof2, kt2
     kt["profiled_ms"] = ms_prof
     rec = room.read_receivers()
     return ms, launches, kt, rec
@@ -369,7 +374,7 @@ def run_rafd(args, rank, world, local_rank):
                 "l2": "inputs larger than L2 (working set %.1f GB/GPU vs 126 MB L2)" % (info["device_bytes"] / 1e9),
                 "timed": "CUDA events on the room stream around K steps replayed from CUDA graphs (the product "
                          "path) after W + %d untimed steps; per-kernel times from K more steps launched with "
-                         "events around every kernel" % GRAPH_WARM,
+                         "events around every kernel (the faster of two such passes)" % GRAPH_WARM,
                 "steps_per_sweep": tb,
                 # RAFD_BENCH_DEVICE pins every rank to one GPU (a functional check of the
                 # multi-rank path): the ranks then share that GPU's bandwidth
