@@ -115,6 +115,7 @@ cudaError_t volume_plan_occupancy(void *plan, const Grid &g, const uint8_t *K, c
 template <typename T>
 cudaError_t volume_plan_create(const Grid &g, void *const u[4], uint8_t *K, int nsm, void **plan);
 void volume_plan_destroy(void *plan);
+void volume_plan_adopt_occupancy(void *dst_plan, void *src_plan);
 // temporal blocking (twostep.cu): the two-step volume kernel over the four
 // field buffers (cur_buf = u^n, prev_buf = u^{n-1} -> out1 = u^{n+1}, out2 =
 // u^{n+2}) and the shell recompute of u^{n+2} (list built by the plan)

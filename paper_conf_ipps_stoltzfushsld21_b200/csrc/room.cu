@@ -1658,9 +1658,7 @@ template <typename T> static int enable_twostep_t(rafd_room *r)
     tr.mark(r->stream, "alloc + memset u[2..3]");
     // the single-step kernel needs TMA maps of the second pair too
     if (rc == RAFD_OK && e == cudaSuccess) e = volume_plan_create<T>(r->g, nu, r->K_alloc, r->nsm, &vp);
-    const char *sk = getenv("RAFD_SKIP_EMPTY");
-    if (rc == RAFD_OK && e == cudaSuccess && !(sk && strcmp(sk, "0") == 0))
-        e = volume_plan_occupancy(vp, r->g, r->K, r->stream);
+    // (the occupancy table is taken over from the current plan at the commit below)
     tr.mark(r->stream, "volume plan");
     if (rc == RAFD_OK && e == cudaSuccess)
         e = twostep_plan_create<T>(r->g, nu, r->K_alloc, r->K, r->idx64, r->nsm, r->stream, &tp, &nsh);
@@ -1679,6 +1677,7 @@ template <typename T> static int enable_twostep_t(rafd_room *r)
     }
     // commit: the cached graphs captured the old plan's arguments
     free_graphs(r);
+    volume_plan_adopt_occupancy(vp, r->vplan);
     volume_plan_destroy(r->vplan);
     r->vplan = vp;
     r->tbplan = tp;
