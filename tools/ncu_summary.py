@@ -40,7 +40,7 @@ def launches(path):
             ns = float(d["Metric Value"]) * (1e3 if d["Metric Unit"] == "usecond" else 1e6 if d["Metric Unit"] == "msecond" else 1)
             per[name].append(ns)
             order.append(name)
-    step = [k for k in per if k.startswith(("k_volume", "k_boundary", "k_src", "k_shell<"))]
+    step = [k for k in per if k.startswith(("k_volume", "k_boundary", "k_src", "k_shell<", "k_shell_bnd<"))]
     tot = sum(sum(per[k]) for k in step)
     out = {"kernels": {}, "note": "ncu --metrics gpu__time_duration.sum --clock-control none: cold-cache, serialised; compare shares"}
     for k in step:
