@@ -133,12 +133,15 @@ template <typename T>
 cudaError_t launch_shell(const void *plan, const Grid &g, const T *u1, const T *u0, const uint8_t *K, T *out,
                          double lambda, cudaStream_t s, bool interior = false);
 // the shell fused with the step-(n+2) boundary update and the source /
-// receivers (whole rooms; the list's node entries must be exactly the room's
-// nodes: twostep_shell_nodes(plan) == Nb)
+// receivers (src_mode as k_boundary's); the list's node entries must be
+// exactly the handle's nodes (twostep_shell_nodes(plan) == Nb).  interior: a
+// slab's interior planes only (list range [sh_lo, sh_hi), nodes
+// [n_first_plane, n_last_start))
 template <typename T>
 cudaError_t launch_shell_bnd(const void *plan, const Grid &g, const T *u1, const T *u0, const uint8_t *K, T *out,
                              double lambda, int MB, const uint8_t *matb, T *ub, T *gst, T *vst, int64_t Nb,
-                             const T *tab, int M, Ctl<T> *ctl, unsigned int *ticket, cudaStream_t s);
+                             const T *tab, int M, Ctl<T> *ctl, unsigned int *ticket, cudaStream_t s,
+                             bool interior = false, int src_mode = 3);
 int64_t twostep_shell_nodes(const void *plan);
 template <typename T>
 cudaError_t launch_boundary(int MB, bool idx64, const void *bpos, const uint8_t *Kb,

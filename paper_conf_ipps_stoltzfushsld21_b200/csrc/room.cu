@@ -912,7 +912,10 @@ static int kernels_per_phase(const rafd_room *r, int phase)
                ((zs == 0 || zs == lnz - 1) ? 1 : 0);
     }
     // interior volume, then either the interior boundary kernel (which runs the
-    // source/receivers in its last block) or k_src_rcv alone
+    // source/receivers in its last block) or k_src_rcv alone; the second
+    // interior phase of a double step (ph 3) is one fused shell + boundary
+    // launch when the slab has interior nodes
+    if (phase == 3 && r->shell_bnd && lnz > 2 && r->n_last_start > r->n_first_plane) return 1;
     return (lnz > 2 ? 1 : 0) + 1;
 }
 
@@ -978,6 +981,15 @@ static cudaError_t enqueue_tb_phase(rafd_room *r, int ph, cudaStream_t s, bool p
         if (e == cudaSuccess && src_edge)
             e = timed(2, [&] { return launch_src_rcv<T>(out, ub, ctl_of<T>(r), s, 1, ms0, ms1); });
     } else {
+        if (lnz > 2 && ph == 3 && r->shell_bnd && bnd_src) {
+            // the interior shell, its boundary nodes and the source / receivers in one pass
+            return timed(3, [&] {
+                return launch_shell_bnd<T>(r->tbplan, g, (const T *)r->u[bC], (const T *)r->u[bB], r->K,
+                                           (T *)r->u[bD], r->lambda, r->MB, r->matb, ub, (T *)r->gst, (T *)r->vst,
+                                           r->nb, (const T *)r->tab, r->M, ctl_of<T>(r), r->ticket, s, true,
+                                           src_edge ? 2 : 3);
+            });
+        }
         if (lnz > 2) {
             if (ph == 1)
                 e = timed(0, [&] {
@@ -1118,11 +1130,12 @@ template <typename T> static int step_t(rafd_room *r, int64_t nsteps)
         return set_err(RAFD_E_CUDA, "step: %s", cudaGetErrorString(e));
     };
     const int64_t kslab = slab ? kernels_per_phase(r, 0) + kernels_per_phase(r, 1) : 0;
+    const int64_t kslab2 = slab ? 2 * kernels_per_phase(r, 0) + kernels_per_phase(r, 1) + kernels_per_phase(r, 3) : 0;
     while (r->tb == 2 && nsteps - done >= 2) {
         cudaError_t e = slab ? slab_step(r, true, r->profiling, r->steps + done)
                              : enqueue_step2<T>(r, r->pair, r->cur, r->stream, r->profiling);
         if (e != cudaSuccess) return slab ? slab_err(e) : set_err(RAFD_E_CUDA, "step: %s", cudaGetErrorString(e));
-        r->launches += slab ? 2 * kslab : kernels_per_double_step(r);
+        r->launches += slab ? kslab2 : kernels_per_double_step(r);
         r->pair ^= 2;
         done += 2;
     }
@@ -1210,7 +1223,7 @@ template <typename T> static int step_group_t(rafd_room **rs, int n, int64_t nst
                 cudaError_t e = slab_phase(r, two, pe + 1, r->stream, r->profiling);
                 if (e != cudaSuccess) return set_err(RAFD_E_CUDA, "step: %s", cudaGetErrorString(e));
                 CK(cudaStreamWaitEvent(r->stream, r->ev_halo, 0));
-                r->launches += kernels_per_phase(r, 1);
+                r->launches += kernels_per_phase(r, two ? pe + 1 : 1);
             }
         }
         for (int k = 0; k < n; k++) {
@@ -1686,8 +1699,7 @@ template <typename T> static int enable_twostep_t(rafd_room *r)
     // room's nodes (always, for a whole room); RAFD_SHELL_BND=0 keeps two passes
     {
         const char *sb = getenv("RAFD_SHELL_BND");
-        r->shell_bnd = r->nranks == 1 && r->nb > 0 && r->scheme == 0 && twostep_shell_nodes(tp) == r->nb &&
-                       !(sb && strcmp(sb, "0") == 0);
+        r->shell_bnd = r->nb > 0 && r->scheme == 0 && twostep_shell_nodes(tp) == r->nb && !(sb && strcmp(sb, "0") == 0);
     }
     r->device_bytes += r->n_shell * (r->idx64 ? 8 : 4) + 56;
     for (int k = 2; k < 4; k++) r->u[k] = nu[k];

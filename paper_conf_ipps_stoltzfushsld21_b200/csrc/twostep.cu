@@ -422,32 +422,42 @@ __global__ void __launch_bounds__(256) k_shell(const IdxT *__restrict__ list, co
 // k_boundary, DESIGN.md §4 order), one store of the final value.  The last
 // block adds the source and records the receivers (as k_boundary).  The
 // source's star entries that are shell voxels are left to their list entry.
+// The list range [lo, hi) (a slab's interior phase: the sub-range of its
+// interior planes, whose node entries are the interior nodes); threads start at
+// the 32-entry group boundary below lo so every warp's ballot covers one whole
+// group (entries below lo are counted, not processed).  Star entries are
+// recomputed only inside the padded planes [zp_lo, zp_hi).  src_mode: as
+// k_boundary's (3: add the source and record receivers; 2: record only).
 template <typename T, int MB, typename IdxT, int ENT>
 __global__ void __launch_bounds__(256)
     k_shell_bnd(const IdxT *__restrict__ list, const uint8_t *__restrict__ nmask, const int64_t *__restrict__ wbase,
-                int64_t n, const int64_t *__restrict__ src, const T *__restrict__ u1, const T *__restrict__ u0,
-                const uint8_t *__restrict__ K, T *__restrict__ out, Grid g, T l2, T l,
+                int64_t lo, int64_t hi, const int64_t *__restrict__ src, const T *__restrict__ u1,
+                const T *__restrict__ u0, const uint8_t *__restrict__ K, T *__restrict__ out, Grid g, T l2, T l,
                 const uint8_t *__restrict__ matb, T *__restrict__ ub, T *__restrict__ gst, T *__restrict__ vst,
-                int64_t Nb, const T *__restrict__ tab, int M, Ctl<T> *ctl, unsigned int *ticket)
+                int64_t Nb, const T *__restrict__ tab, int M, Ctl<T> *ctl, unsigned int *ticket, int zp_lo,
+                int zp_hi, int src_mode)
 {
     using R = rn<T>;
     const int lane = threadIdx.x & 31;
+    const int64_t lo32 = lo & ~(int64_t)31, nrange = hi - lo32;
     // ENT entries per thread (entry = block * 256 * ENT + e * 256 + tid): each
     // warp still covers 32 consecutive entries per e, and the block's ticket
     // below is paid once per 256 * ENT entries
 #pragma unroll
     for (int e = 0; e < ENT; e++) {
-        const int64_t i = (int64_t)blockIdx.x * (256 * ENT) + e * 256 + threadIdx.x;
-        const bool in_list = i < n;
+        const int64_t j = (int64_t)blockIdx.x * (256 * ENT) + e * 256 + threadIdx.x;
+        const int64_t i = lo32 + j;  // list index of a list thread
+        const bool in_list = j < nrange;
         int64_t p = -1;
         uint32_t m = 0;
         int nbr = 0;
         if (in_list) {
-            p = (int64_t)list[i];
             m = nmask[i];
             nbr = __popc(m);
-        } else if (i < n + 7) {
-            p = src[i - n];
+            if (i >= lo) p = (int64_t)list[i];
+        } else if (j < nrange + 7) {
+            p = src[j - nrange];
+            if (p >= 0 && (p < (int64_t)zp_lo * g.plane || p >= (int64_t)zp_hi * g.plane)) p = -1;
             if (p >= 0) {  // a star voxel: recomputed here unless it is a shell voxel (its list entry does it)
                 const int64_t d[6] = {-1, 1, -g.pitch, g.pitch, -g.plane, g.plane};
                 nbr = K[p];
@@ -464,6 +474,7 @@ __global__ void __launch_bounds__(256)
         const bool node = in_list && nbr < 6;
         const unsigned bal = __ballot_sync(0xffffffffu, node);
         const int64_t rank = node ? wbase[i >> 5] + __popc(bal & ((1u << lane) - 1u)) : 0;
+        if (p < 0) continue;  // below lo, or a star voxel left to its list entry
         if (p >= 0) {
             T uprev = (T)0, gb[MB > 0 ? MB : 1], vb[MB > 0 ? MB : 1];
             int mi = 0;
@@ -512,7 +523,7 @@ __global__ void __launch_bounds__(256)
     __syncthreads();
     if (last) {
         __threadfence();
-        src_rcv_block<T>(out, ub, ctl, 3, 0, 0, cb);
+        src_rcv_block<T>(out, ub, ctl, src_mode, 0, 0, cb);
         if (threadIdx.x == 0) *ticket = 0u;
     }
 }
@@ -788,31 +799,37 @@ static constexpr int kShellEnt = 1;  // entries per thread of k_shell_bnd
 template <typename T, int MB>
 static cudaError_t launch_sb(const TwoStepPlan *pl, const Grid &g, const T *u1, const T *u0, const uint8_t *K,
                              T *out, T l2, T l, const uint8_t *matb, T *ub, T *gst, T *vst, int64_t Nb, const T *tab,
-                             int M, Ctl<T> *ctl, unsigned int *ticket, cudaStream_t s)
+                             int M, Ctl<T> *ctl, unsigned int *ticket, cudaStream_t s, int64_t lo, int64_t hi,
+                             int zp_lo, int zp_hi, int src_mode)
 {
-    const int64_t n = pl->n_shell;
     constexpr int ENT = kShellEnt;
+    const int64_t n = hi - (lo & ~(int64_t)31);
     const unsigned blocks = (unsigned)((n + 7 + 256 * ENT - 1) / (256 * ENT));
     if (pl->idx64)
-        k_shell_bnd<T, MB, int64_t, ENT><<<blocks, 256, 0, s>>>((const int64_t *)pl->list, pl->nmask, pl->wbase, n, pl->src,
-                                                           u1, u0, K, out, g, l2, l, matb, ub, gst, vst, Nb, tab, M,
-                                                           ctl, ticket);
+        k_shell_bnd<T, MB, int64_t, ENT><<<blocks, 256, 0, s>>>((const int64_t *)pl->list, pl->nmask, pl->wbase, lo, hi,
+                                                               pl->src, u1, u0, K, out, g, l2, l, matb, ub, gst, vst,
+                                                               Nb, tab, M, ctl, ticket, zp_lo, zp_hi, src_mode);
     else
-        k_shell_bnd<T, MB, uint32_t, ENT><<<blocks, 256, 0, s>>>((const uint32_t *)pl->list, pl->nmask, pl->wbase, n,
-                                                            pl->src, u1, u0, K, out, g, l2, l, matb, ub, gst, vst, Nb,
-                                                            tab, M, ctl, ticket);
+        k_shell_bnd<T, MB, uint32_t, ENT><<<blocks, 256, 0, s>>>((const uint32_t *)pl->list, pl->nmask, pl->wbase, lo,
+                                                                hi, pl->src, u1, u0, K, out, g, l2, l, matb, ub, gst,
+                                                                vst, Nb, tab, M, ctl, ticket, zp_lo, zp_hi, src_mode);
     return cudaGetLastError();
 }
 
 template <typename T>
 cudaError_t launch_shell_bnd(const void *plan, const Grid &g, const T *u1, const T *u0, const uint8_t *K, T *out,
                              double lambda, int MB, const uint8_t *matb, T *ub, T *gst, T *vst, int64_t Nb,
-                             const T *tab, int M, Ctl<T> *ctl, unsigned int *ticket, cudaStream_t s)
+                             const T *tab, int M, Ctl<T> *ctl, unsigned int *ticket, cudaStream_t s, bool interior,
+                             int src_mode)
 {
     const auto *pl = (const TwoStepPlan *)plan;
     const T l2 = (T)(lambda * lambda), l = (T)lambda;
+    if (interior && g.lnz < 3) return cudaSuccess;
+    const int64_t lo = interior ? pl->sh_lo : 0, hi = interior ? pl->sh_hi : pl->n_shell;
+    const int zp_lo = interior ? 2 : 1, zp_hi = interior ? g.lnz : g.lnz + 1;
 #define RAFD_SB(k) \
-    case k: return launch_sb<T, k>(pl, g, u1, u0, K, out, l2, l, matb, ub, gst, vst, Nb, tab, M, ctl, ticket, s);
+    case k:        \
+        return launch_sb<T, k>(pl, g, u1, u0, K, out, l2, l, matb, ub, gst, vst, Nb, tab, M, ctl, ticket, s, lo, hi, zp_lo, zp_hi, src_mode);
     switch (MB) {
         RAFD_SB(0)
         RAFD_SB(1)
@@ -837,7 +854,7 @@ cudaError_t launch_shell_bnd(const void *plan, const Grid &g, const T *u1, const
                                          double, cudaStream_t, bool);                                                 \
     template cudaError_t launch_shell_bnd<T>(const void *, const Grid &, const T *, const T *, const uint8_t *, T *, \
                                              double, int, const uint8_t *, T *, T *, T *, int64_t, const T *, int,   \
-                                             Ctl<T> *, unsigned int *, cudaStream_t);
+                                             Ctl<T> *, unsigned int *, cudaStream_t, bool, int);
 RAFD_TB_INST(float)
 RAFD_TB_INST(double)
 #undef RAFD_TB_INST
