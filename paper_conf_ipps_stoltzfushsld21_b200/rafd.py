@@ -133,9 +133,9 @@ class RafdError(RuntimeError):
         self.code = code
 
 
-def _check(rc):
+def _check(rc, L=None):
     if rc != RAFD_OK:
-        raise RafdError(rc, lib().rafd_last_error().decode())
+        raise RafdError(rc, (L or lib()).rafd_last_error().decode())
 
 
 def _addr(a):
@@ -161,6 +161,10 @@ class Room:
                  device=0, stream=None, rank=0, nranks=1, nccl_id=None, z_begin=0, z_end=0,
                  mask_z0=0, dims=None, scheme=0, loss1=1.0, loss2=1.0):
         L = lib()
+        # the handle belongs to this library: every method (and __del__) calls
+        # it, even if the module is later pointed at another build (RAFD_LIB /
+        # the oracle's librafd_oracle.so in tests)
+        self._L = L
         # dims = (nx, ny, nz) of the room when `mask` holds only planes [mask_z0, ...)
         nz, ny, nx = (int(s) for s in mask.shape)
         if dims is not None:
@@ -193,7 +197,7 @@ class Room:
                            None if idbuf is None else C.addressof(idbuf), int(z_begin), int(z_end),
                            int(mask_z0), int(scheme), float(loss1), float(loss2))
         h = C.c_void_p()
-        _check(L.rafd_create(C.byref(d), C.byref(h)))
+        _check(L.rafd_create(C.byref(d), C.byref(h)), L)
         self.h = h
         self._keep = (mask, matmap, beta0, Dd, Ed, Fd)
         self.shape = (nz, ny, nx)
@@ -208,7 +212,7 @@ class Room:
     # --- lifetime
     def destroy(self):
         if getattr(self, "h", None):
-            lib().rafd_destroy(self.h)
+            self._L.rafd_destroy(self.h)
             self.h = None
 
     def __del__(self):
@@ -220,12 +224,12 @@ class Room:
     # --- set
     def set_source(self, xyz, sig):
         sig = _f64(sig).reshape(-1)
-        _check(lib().rafd_set_source(self.h, int(xyz[0]), int(xyz[1]), int(xyz[2]),
+        _check(self._L.rafd_set_source(self.h, int(xyz[0]), int(xyz[1]), int(xyz[2]),
                                      sig.ctypes.data, sig.size))
 
     def set_receivers(self, xyzs):
         a = np.ascontiguousarray(np.asarray(xyzs, dtype=np.int32).reshape(-1, 3))
-        _check(lib().rafd_set_receivers(self.h, a.shape[0], a.ctypes.data))
+        _check(self._L.rafd_set_receivers(self.h, a.shape[0], a.ctypes.data))
         self.nrcv = a.shape[0]
 
     def set_state(self, u_prev=None, u_curr=None, v=None, g=None):
@@ -234,21 +238,21 @@ class Room:
                 return a
             return np.ascontiguousarray(a, dtype=self.dtype)
         arrs = [conv(a) for a in (u_prev, u_curr, v, g)]
-        _check(lib().rafd_set_state(self.h, *[_addr(a) for a in arrs]))
+        _check(self._L.rafd_set_state(self.h, *[_addr(a) for a in arrs]))
 
     def set_step(self, n):
-        _check(lib().rafd_set_step(self.h, int(n)))
+        _check(self._L.rafd_set_step(self.h, int(n)))
 
     # --- run
     def step(self, n):
-        _check(lib().rafd_step(self.h, int(n)))
+        _check(self._L.rafd_step(self.h, int(n)))
 
     def set_temporal_blocking(self, steps_per_sweep):
         """rafd_set_temporal_blocking: 2 = two leapfrog steps per grid sweep."""
-        _check(lib().rafd_set_temporal_blocking(self.h, int(steps_per_sweep)))
+        _check(self._L.rafd_set_temporal_blocking(self.h, int(steps_per_sweep)))
 
     def synchronize(self):
-        _check(lib().rafd_synchronize(self.h))
+        _check(self._L.rafd_synchronize(self.h))
 
     # --- read
     def read_receivers(self, cap=None):
@@ -258,7 +262,7 @@ class Room:
             cap = max(1, self.get_info()["steps"])
         out = np.zeros((self.nrcv, cap), dtype=np.float64)
         n = C.c_int64()
-        _check(lib().rafd_read_receivers(self.h, out.ctypes.data, cap, C.byref(n)))
+        _check(self._L.rafd_read_receivers(self.h, out.ctypes.data, cap, C.byref(n)))
         return out[:, : n.value].copy()
 
     def read_field(self, out_curr=None, out_prev=None):
@@ -268,14 +272,14 @@ class Room:
         shp = (lnz, self.shape[1], self.shape[2])
         cur = np.zeros(shp, dtype=self.dtype) if out_curr is None else out_curr
         prv = np.zeros(shp, dtype=self.dtype) if out_prev is None else out_prev
-        _check(lib().rafd_read_field(self.h, None if cur is False else _addr(cur),
+        _check(self._L.rafd_read_field(self.h, None if cur is False else _addr(cur),
                                      None if prv is False else _addr(prv)))
         return (None if cur is False else cur), (None if prv is False else prv)
 
     def read_branch_state(self):
         v = np.zeros((self.MB, self.nb), dtype=self.dtype)
         g = np.zeros((self.MB, self.nb), dtype=self.dtype)
-        _check(lib().rafd_read_branch_state(self.h, _addr(v), _addr(g)))
+        _check(self._L.rafd_read_branch_state(self.h, _addr(v), _addr(g)))
         return v, g
 
     def get_classification(self):
@@ -284,49 +288,49 @@ class Room:
         bidx = np.zeros(self.nb, dtype=np.int64)
         Kb = np.zeros(self.nb, dtype=np.uint8)
         matb = np.zeros(self.nb, dtype=np.uint8)
-        _check(lib().rafd_get_classification(self.h, K.ctypes.data, bidx.ctypes.data,
+        _check(self._L.rafd_get_classification(self.h, K.ctypes.data, bidx.ctypes.data,
                                              Kb.ctypes.data, matb.ctypes.data))
         return K, bidx, Kb, matb
 
     def get_info(self):
         i = rafd_info()
-        _check(lib().rafd_get_info(self.h, C.byref(i)))
+        _check(self._L.rafd_get_info(self.h, C.byref(i)))
         d = {k: getattr(i, k) for k, _ in rafd_info._fields_}
         d["k_hist"] = list(i.k_hist)
         return d
 
     def energy(self):
         h = C.c_double()
-        _check(lib().rafd_energy(self.h, C.byref(h)))
+        _check(self._L.rafd_energy(self.h, C.byref(h)))
         return h.value
 
     def set_profiling(self, on=True):
-        _check(lib().rafd_set_profiling(self.h, 1 if on else 0))
+        _check(self._L.rafd_set_profiling(self.h, 1 if on else 0))
 
     def get_kernel_times(self):
         t = rafd_kernel_times()
-        _check(lib().rafd_get_kernel_times(self.h, C.byref(t)))
+        _check(self._L.rafd_get_kernel_times(self.h, C.byref(t)))
         return {k: getattr(t, k) for k, _ in rafd_kernel_times._fields_}
 
     def ipc_handle(self):
         """This slab's IPC blob (bytes) for rafd_ipc_connect of its neighbours."""
         buf = (C.c_uint8 * RAFD_IPC_BLOB_BYTES)()
-        _check(lib().rafd_ipc_handle(self.h, buf))
+        _check(self._L.rafd_ipc_handle(self.h, buf))
         return bytes(buf)
 
     def ipc_connect(self, lower, upper):
         lo = None if lower is None else (C.c_uint8 * RAFD_IPC_BLOB_BYTES).from_buffer_copy(lower)
         hi = None if upper is None else (C.c_uint8 * RAFD_IPC_BLOB_BYTES).from_buffer_copy(upper)
-        _check(lib().rafd_ipc_connect(self.h, None if lo is None else C.addressof(lo),
+        _check(self._L.rafd_ipc_connect(self.h, None if lo is None else C.addressof(lo),
                                       None if hi is None else C.addressof(hi)))
 
     def set_halo_push(self, on=True):
         """rafd_set_halo_push: the edge-phase kernels store the halo into the
         neighbours' ghost planes (device-initiated) instead of copy pulls."""
-        _check(lib().rafd_set_halo_push(self.h, int(bool(on))))
+        _check(self._L.rafd_set_halo_push(self.h, int(bool(on))))
 
     def launch_count(self):
-        return int(lib().rafd_launch_count(self.h))
+        return int(self._L.rafd_launch_count(self.h))
 
 
 # ------------------------------------------------------------------ C-ABI names

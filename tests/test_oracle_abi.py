@@ -108,6 +108,7 @@ def test_errors_through_the_abi(orc):
         with pytest.raises(rafd.RafdError) as e:
             rafd.Room(mask, LAM, 32, beta0, D, E, F, matmap=mm, rank=0, nranks=2, z_begin=0, z_end=9)
         assert e.value.code == rafd.RAFD_E_STATE
+        r.destroy()
 
 
 @pytest.mark.parametrize("dims,p", [((21, 17, 40), 3), ((9, 8, 33), 5)])
