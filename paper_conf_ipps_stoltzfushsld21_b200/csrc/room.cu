@@ -334,11 +334,6 @@ template <typename T> static int create_t(rafd_room *r, const rafd_room_desc *d)
     g.xo = (int)(128 / sizeof(T));
     const int64_t align = 128 / (int64_t)sizeof(T);
     g.pitch = ((g.xo + r->nx + 1 + align - 1) / align) * align;
-    {
-        // RAFD_PITCH_PAD: extra 128-byte lines per row (DRAM channel-mapping experiment)
-        const char *e = getenv("RAFD_PITCH_PAD");
-        if (e) g.pitch += (int64_t)atoi(e) * align;
-    }
     g.plane = g.pitch * (r->ny + 2);
     g.total = g.plane * (g.lnz + 2);
     r->idx64 = g.total >= (int64_t)UINT32_MAX;

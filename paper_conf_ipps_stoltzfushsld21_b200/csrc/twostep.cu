@@ -32,8 +32,6 @@
 
 #include <stdlib.h>
 
-#include <type_traits>
-
 #include "bnd_math.cuh"
 #include "internal.cuh"
 
@@ -49,10 +47,6 @@ static __device__ __forceinline__ void mbar_init(uint64_t *b, uint32_t count)
 static __device__ __forceinline__ void mbar_expect_tx(uint64_t *b, uint32_t bytes)
 {
     asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(b)), "r"(bytes) : "memory");
-}
-static __device__ __forceinline__ void mbar_arrive(uint64_t *b)
-{
-    asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(b)) : "memory");
 }
 static __device__ __forceinline__ void mbar_wait(uint64_t *b, uint32_t parity)
 {
@@ -79,53 +73,11 @@ static __device__ __forceinline__ uint64_t policy_evict_first()
     asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p));
     return p;
 }
-// store policy of the two-step kernels (RAFD_TB_STPOL experiment: 0 evict_first
-// (default), 1 evict_normal, 2 evict_last, 3 evict_unchanged)
-__constant__ int c_tb_stpol = 0;
-static __device__ __forceinline__ uint64_t policy_store()
-{
-    uint64_t p;
-    const int v = c_tb_stpol;
-    if (v == 1)
-        asm volatile("createpolicy.fractional.L2::evict_normal.b64 %0, 1.0;" : "=l"(p));
-    else if (v == 2)
-        asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(p));
-    else if (v == 3)
-        asm volatile("createpolicy.fractional.L2::evict_unchanged.b64 %0, 1.0;" : "=l"(p));
-    else
-        asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p));
-    return p;
-}
 static __device__ __forceinline__ void st_v4_hint(void *ptr, uint4 v, uint64_t pol)
 {
     asm volatile("st.global.L2::cache_hint.v4.b32 [%0], {%1, %2, %3, %4}, %5;" ::"l"(ptr), "r"(v.x), "r"(v.y),
                  "r"(v.z), "r"(v.w), "l"(pol)
                  : "memory");
-}
-// TMA store of a box from shared memory (bulk-group completion), L2 evict-first
-static __device__ __forceinline__ void tma_store_3d(const CUtensorMap *map, const void *src, int c0, int c1, int c2,
-                                                    uint64_t pol)
-{
-    asm volatile(
-        "cp.async.bulk.tensor.3d.global.shared::cta.tile.bulk_group.L2::cache_hint [%0, {%1, %2, %3}], [%4], %5;" ::"l"(
-            (uint64_t)map),
-        "r"(c0), "r"(c1), "r"(c2), "r"(smem_u32(src)), "l"(pol)
-        : "memory");
-}
-static __device__ __forceinline__ void bulk_commit() { asm volatile("cp.async.bulk.commit_group;" ::: "memory"); }
-template <int N> static __device__ __forceinline__ void bulk_wait_read()
-{
-    asm volatile("cp.async.bulk.wait_group.read %0;" ::"n"(N) : "memory");
-}
-static __device__ __forceinline__ void bulk_wait_all() { asm volatile("cp.async.bulk.wait_group 0;" ::: "memory"); }
-static __device__ __forceinline__ void fence_proxy_async() { asm volatile("fence.proxy.async.shared::cta;" ::: "memory"); }
-// p + d elements, opaque to the compiler (keeps a running pointer in registers
-// instead of re-deriving it from the plane index every iteration)
-template <typename T> static __device__ __forceinline__ T *advance(T *p, int64_t d)
-{
-    uint64_t r;
-    asm volatile("add.s64 %0, %1, %2;" : "=l"(r) : "l"((uint64_t)p), "l"(d * (int64_t)sizeof(T)));
-    return (T *)r;
 }
 }  // namespace tb
 
@@ -232,7 +184,7 @@ __global__ void __launch_bounds__(TbGeom<T, TY, SU, SP>::NT, 1)
     }
     __syncthreads();
     uint32_t uph = 0, pph = 0;
-    const uint64_t pol = tb::policy_store();
+    const uint64_t pol = tb::policy_evict_first();
 
     // stored planes: local [z_lo, z_hi) (a z slab stores its interior planes;
     // the u^n ghost planes it reads are the neighbours' edge planes)
@@ -398,468 +350,6 @@ __global__ void __launch_bounds__(TbGeom<T, TY, SU, SP>::NT, 1)
     if (DYN && tid == 0) {
         __threadfence();
         if (atomicAdd(work + 1, 1u) == gridDim.x - 1) {  // every CTA has taken its last unit
-            atomicExch(work, 0u);
-            atomicExch(work + 1, 0u);
-        }
-    }
-}
-
-// ------------------------------------------------------------------ k_volume2w
-// The same two-step sweep (same tiles, same TMA boxes, same arithmetic, so the
-// same bits), organised for more warps and fewer instructions per update:
-//  * one core row per warp (TY warps, 32 x TY threads; warps 0 and TY-1 also
-//    compute the step-(n+1) halo rows -1 and TY), so an SM holds 32 warps
-//    instead of 17 to hide shared-memory and barrier latency;
-//  * no register windows: every z-neighbour comes from shared memory -- u^n
-//    planes q-1, q, q+1 from a 5-slot TMA ring, u^{n+1} planes q-2, q-1 from a
-//    3-slot ring -- so the loop carries one K word per thread;
-//  * step n+2 of plane q-1 reads u^{n+1} only from slots written in earlier
-//    iterations (its z+1 neighbour, u^{n+1}(q), is the thread's own step-(n+1)
-//    result) and a warp's reads of the oldest slot are of its own row, so the
-//    only cross-warp hazards per plane are "neighbour rows of u^{n+1}(q-1)
-//    written" (RAW) and "every warp done with the slots the TMA refills" (WAR).
-// Synchronisation (template bit SPLIT): either one CTA barrier per plane, or a
-// split barrier -- every thread arrives on an mbarrier when its plane is done
-// and waits for the previous plane's phase only before its step n+2, so a warp
-// runs its next step n+1 while the slowest warp finishes; the TMA issuer
-// refills the slots the previous plane freed right after that wait.
-// Template bit RUNPTR: store addresses kept as running pointers (one 64-bit add
-// per plane) instead of derived from the plane index at each store.
-template <typename T, int TY> struct TbRowGeom {
-    using B = TbGeom<T, TY, 4, 4>;  // box shapes (the plan's tensor maps)
-    static constexpr int VEC = B::VEC, TX = B::TX, TXO = B::TXO, UROW = B::UROW, UR = B::UR, PR = B::PR;
-    static constexpr int KROW = B::KROW, U_BYTES = B::U_BYTES, P_BYTES = B::P_BYTES, K_BYTES = B::K_BYTES;
-    static constexpr int U1_BYTES = B::U1_BYTES, U_TX = B::U_TX, PK_TX = B::PK_TX;
-    static constexpr int SU = 5, SP = 3, S1 = 3;
-    static constexpr int NW = TY, NT = 32 * TY;
-    static constexpr int SMEM = SU * U_BYTES + SP * (P_BYTES + K_BYTES) + S1 * U1_BYTES + (SU + SP + 1) * 8 + 128;
-};
-
-static __device__ __forceinline__ int ring_next(int s, int n) { return s + 1 == n ? 0 : s + 1; }
-
-template <typename T, int TY, bool DYN, int V>
-__global__ void __launch_bounds__(TbRowGeom<T, TY>::NT, 1)
-    k_volume2w(const __grid_constant__ CUtensorMap umap, const __grid_constant__ CUtensorMap pmap,
-               const __grid_constant__ CUtensorMap kmap, T *__restrict__ out1, T *__restrict__ out2, Grid g, T l2,
-               int z_lo, int z_hi, int zchunk, int tiles_x, int tiles_y, unsigned int *work)
-{
-    using G = TbRowGeom<T, TY>;
-    using KW = typename Vec16<T>::K;
-    constexpr bool SPLIT = (V & 1) != 0, RUNPTR = (V & 2) != 0;
-    constexpr int VEC = G::VEC, TX = G::TX, TXO = G::TXO, UROW = G::UROW, SU = G::SU, SP = G::SP;
-    constexpr int UE = G::U_BYTES / (int)sizeof(T), PE = G::P_BYTES / (int)sizeof(T), U1E = G::U1_BYTES / (int)sizeof(T);
-    extern __shared__ __align__(1024) unsigned char smem_raw[];
-    unsigned char *const base = smem_raw;
-    T *us = (T *)base;                                                  // SU u^n slots
-    T *ps = (T *)(base + SU * G::U_BYTES);                              // SP u^{n-1} slots
-    uint8_t *ks = base + SU * G::U_BYTES + SP * G::P_BYTES;             // SP K slots
-    T *u1s = (T *)(base + SU * G::U_BYTES + SP * (G::P_BYTES + G::K_BYTES));  // 3 u^{n+1} planes
-    uint64_t *bar = (uint64_t *)((unsigned char *)u1s + G::S1 * G::U1_BYTES);
-    uint64_t *done = bar + SU + SP;  // split barrier: every thread arrives once per plane
-    int *const s_next = (int *)(done + 1);
-    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-    constexpr int ISSUER = 32;  // warp 1, lane 0 issues the TMA loads (warps 0 and TY-1 carry the halo rows)
-
-    if (tid == 0) {
-        if (tb::smem_u32(smem_raw) & 127u) __trap();
-        for (int i = 0; i < SU + SP; i++) tb::mbar_init(&bar[i], 1);
-        tb::mbar_init(done, G::NT);
-        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-    }
-    __syncthreads();
-    uint32_t uph = 0, pph = 0;
-    uint32_t narr = 0;  // this thread's arrivals on `done` (= planes processed)
-    const uint64_t pol = tb::policy_store();
-
-    const int nz = z_hi - z_lo;
-    const int nchunks = (nz + zchunk - 1) / zchunk;
-    const int tiles = tiles_x * tiles_y;
-    const int units = nchunks * tiles;
-    const int r = warp;  // this warp's core row
-    const int col = VEC + lane * VEC;
-    const int hcol = lane == 0 ? VEC - 1 : VEC + TX;  // x halo of lanes 0 / 31 in a u^n smem row
-    int unit = blockIdx.x, next_unit = 0;
-    if constexpr (DYN) {
-        if (tid == 0) *s_next = (int)atomicAdd(work, 1u);
-        __syncthreads();
-        unit = *s_next;
-    }
-    while (unit < units) {
-        if constexpr (DYN) {
-            if (tid == 0) next_unit = (int)atomicAdd(work, 1u);
-        }
-        const int chunk = unit / tiles, t = unit % tiles;
-        const int ty = t / tiles_x, tx = t % tiles_x;
-        const int pa = 1 + z_lo + chunk * zchunk;
-        const int pb = min(1 + z_hi, pa + zchunk);
-        const int ox = tx * TXO, oy = ty * TY;
-        const int ux = g.xo + ox - 2 * VEC, uy = oy - 1;
-        const int px = g.xo + ox - VEC, py = oy;
-        const int kx = px + k_shift(g);
-        const int kd = kx & 15;
-        // ring slots: u^n plane p in slot (p - (pa-2)) mod SU, u^{n-1}/K plane p
-        // in slot (p - (pa-1)) mod SP, u^{n+1} plane p in slot (p - (pa-1)) mod 3
-        auto issue_u = [&](int p, int s) {
-            tb::mbar_expect_tx(&bar[s], G::U_TX);
-            tb::tma_load_3d((unsigned char *)us + s * G::U_BYTES, &umap, &bar[s], ux, uy, p);
-        };
-        auto issue_pk = [&](int p, int s) {
-            tb::mbar_expect_tx(&bar[SU + s], G::PK_TX);
-            tb::tma_load_3d((unsigned char *)ps + s * G::P_BYTES, &pmap, &bar[SU + s], px, py, p);
-            tb::tma_load_3d(ks + s * G::K_BYTES, &kmap, &bar[SU + s], kx - kd, py, p);
-        };
-        auto wait_u = [&](int s) {
-            tb::mbar_wait(&bar[s], (uph >> s) & 1);
-            uph ^= 1u << s;
-        };
-        auto wait_pk = [&](int s) {
-            tb::mbar_wait(&bar[SU + s], (pph >> s) & 1);
-            pph ^= 1u << s;
-        };
-        __syncthreads();  // the previous unit is done with every slot
-        if (tid == ISSUER) {
-            asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-            for (int i = 0; i < SU && pa - 2 + i <= pb + 1; i++) issue_u(pa - 2 + i, i);
-            for (int i = 0; i < SP && pa - 1 + i <= pb; i++) issue_pk(pa - 1 + i, i);
-        }
-        int su_mm = SU - 1;                 // u^n slot of plane q-2 (split: refilled in iteration q)
-        int su_m = 0, su_c = 1, su_p = 2;  // u^n slots of planes q-1, q, q+1
-        int sp_m = SP - 1, sp_c = 0;        // u^{n-1}/K slots of planes q-1, q
-        int s1_c = 0, s1_m = 2, s1_mm = 1;  // u^{n+1} slots of planes q, q-1, q-2
-        wait_u(su_m);
-        wait_u(su_c);
-        KW km = 0;  // K of plane q-1 at this thread's core vector
-        const bool lane_core = lane >= 1 && lane <= 30;
-        const int xv = ox + (lane - 1) * VEC;
-        const bool x_ok = lane_core && xv < g.nx;
-        const bool y_ok = oy + r < g.ny;
-        const bool st_ok = x_ok && y_ok;
-        const int64_t roff = (int64_t)(oy + r + 1) * g.pitch + g.xo + xv;
-        T *dst1 = out1 + ((int64_t)(pa - 1) * g.plane + roff);  // RUNPTR: plane q (u^{n+1})
-        T *dst2 = out2 + ((int64_t)(pa - 2) * g.plane + roff);  // RUNPTR: plane q-1 (u^{n+2})
-        for (int q = pa - 1; q <= pb; q++) {
-            wait_u(su_p);
-            wait_pk(sp_c);
-            const T *uqm = us + su_m * UE, *uq = us + su_c * UE, *uqp = us + su_p * UE;
-            const T *pq = ps + sp_c * PE;
-            const uint8_t *kq = ks + sp_c * G::K_BYTES;
-            T *u1w = u1s + s1_c * U1E;
-            // step n+1 on plane q at step row rr (-1 .. TY): u^{n+1} to shared
-            // memory; zm = u^n(q-1) is returned (step n+2's u^{n-1} at row r)
-            auto step1 = [&](int rr, T *o1, T *zm) -> KW {
-                const int sr = rr + 2;
-                T c[VEC], ym[VEC], yp[VEC], zp[VEC], pv[VEC];
-                *(uint4 *)c = *(const uint4 *)(uq + sr * UROW + col);
-                *(uint4 *)ym = *(const uint4 *)(uq + (sr - 1) * UROW + col);
-                *(uint4 *)yp = *(const uint4 *)(uq + (sr + 1) * UROW + col);
-                *(uint4 *)zm = *(const uint4 *)(uqm + sr * UROW + col);
-                *(uint4 *)zp = *(const uint4 *)(uqp + sr * UROW + col);
-                *(uint4 *)pv = *(const uint4 *)(pq + (rr + 1) * TX + lane * VEC);
-                const KW kw = *(const KW *)(kq + (rr + 1) * G::KROW + kd + lane * VEC);
-                const T halo = uq[sr * UROW + hcol];
-                T left = __shfl_up_sync(0xffffffffu, c[VEC - 1], 1);
-                T right = __shfl_down_sync(0xffffffffu, c[0], 1);
-                left = lane == 0 ? halo : left;
-                right = lane == 31 ? halo : right;
-                vol_vec<T>(c, ym, yp, zm, zp, pv, left, right, (uint32_t)kw, l2, o1);
-                *(uint4 *)(u1w + (rr + 1) * TX + lane * VEC) = *(const uint4 *)o1;
-                return kw;
-            };
-            T o1[VEC], zmv[VEC];
-            const KW kc = step1(r, o1, zmv);
-            if constexpr (RUNPTR) {
-                if (q >= pa && q < pb && st_ok) tb::st_v4_hint(dst1, *(const uint4 *)o1, pol);
-            } else {
-                if (q >= pa && q < pb && st_ok)
-                    tb::st_v4_hint(out1 + (int64_t)q * g.plane + roff, *(const uint4 *)o1, pol);
-            }
-            if (warp == 0 || warp == TY - 1) {  // the halo rows (u^{n+1} to shared memory only)
-                T oh[VEC], zh[VEC];
-                step1(warp == 0 ? -1 : TY, oh, zh);
-            }
-            if constexpr (SPLIT) {
-                // every thread has finished plane q-1: its u^{n+1} rows are
-                // written and the slots of u^n(q-2), u^{n-1}/K(q-1) are free
-                if (q >= pa) {
-                    tb::mbar_wait(done, (narr - 1u) & 1u);  // the phase of plane q-1
-                    if (tid == ISSUER) {
-                        asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-                        if (q - 2 + SU <= pb + 1) issue_u(q - 2 + SU, su_mm);
-                        if (q - 1 + SP <= pb) issue_pk(q - 1 + SP, sp_m);
-                    }
-                }
-            }
-            // step n+2 on plane q-1, row r: u^{n+1}(q-1) from shared memory (rows
-            // r-1..r+1), u^{n+1}(q-2) from the slot before, u^{n+1}(q) = o1
-            if (q - 1 >= pa) {
-                const T *u1r = u1s + s1_m * U1E, *u1rr = u1s + s1_mm * U1E;
-                T c[VEC], ym[VEC], yp[VEC], zm[VEC], o2[VEC];
-                *(uint4 *)c = *(const uint4 *)(u1r + (r + 1) * TX + lane * VEC);
-                *(uint4 *)ym = *(const uint4 *)(u1r + r * TX + lane * VEC);
-                *(uint4 *)yp = *(const uint4 *)(u1r + (r + 2) * TX + lane * VEC);
-                *(uint4 *)zm = *(const uint4 *)(u1rr + (r + 1) * TX + lane * VEC);
-                const T left = __shfl_up_sync(0xffffffffu, c[VEC - 1], 1);
-                const T right = __shfl_down_sync(0xffffffffu, c[0], 1);
-                vol_vec<T>(c, ym, yp, zm, o1, zmv, left, right, (uint32_t)km, l2, o2);
-                if constexpr (RUNPTR) {
-                    if (st_ok) tb::st_v4_hint(dst2, *(const uint4 *)o2, pol);
-                } else {
-                    if (st_ok) tb::st_v4_hint(out2 + (int64_t)(q - 1) * g.plane + roff, *(const uint4 *)o2, pol);
-                }
-            }
-            km = kc;
-            if constexpr (SPLIT) {
-                tb::mbar_arrive(done);  // plane q done (its reads and its u^{n+1} row)
-                narr++;
-            } else {
-                __syncthreads();  // u^n(q-1), u^{n-1}/K(q), u^{n+1}(q-2) no longer read
-                if (tid == ISSUER) {
-                    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-                    if (q - 1 + SU <= pb + 1) issue_u(q - 1 + SU, su_m);
-                    if (q + SP <= pb) issue_pk(q + SP, sp_c);
-                }
-            }
-            if constexpr (RUNPTR) {
-                dst1 = tb::advance(dst1, g.plane);
-                dst2 = tb::advance(dst2, g.plane);
-            }
-            su_mm = su_m;
-            su_m = su_c;
-            su_c = su_p;
-            su_p = ring_next(su_p, SU);
-            sp_m = sp_c;
-            sp_c = ring_next(sp_c, SP);
-            s1_mm = s1_m;
-            s1_m = s1_c;
-            s1_c = ring_next(s1_c, 3);
-        }
-        if constexpr (DYN) {
-            if (tid == 0) *s_next = next_unit;
-            __syncthreads();
-            unit = *s_next;
-        } else {
-            unit += gridDim.x;
-        }
-    }
-    if (DYN && tid == 0) {
-        __threadfence();
-        if (atomicAdd(work + 1, 1u) == gridDim.x - 1) {
-            atomicExch(work, 0u);
-            atomicExch(work + 1, 0u);
-        }
-    }
-}
-
-// ------------------------------------------------------------------ k_volume2u
-// The same two-step sweep (same tiles, same TMA boxes, same arithmetic, so the
-// same bits), organised for more warps and fewer instructions per update:
-//  * one step-(n+1) row per warp (TY + 2 = 32 warps, rows -1 .. TY; warps
-//    1 .. TY also do step n+2 of their row), so an SM holds 32 warps instead
-//    of 17 to hide shared-memory and barrier latency;
-//  * rings of 4 u^n and 4 u^{n-1}/K slots and a plane loop unrolled by 4, so
-//    every slot address is a compile-time offset; the u^n z-1 neighbour of a
-//    row is the thread's centre vector of the previous plane (registers), so a
-//    u^n slot is free as soon as its plane has been the centre plane;
-//  * u^{n+1} in a 3-slot shared ring: step n+2 of plane q-1 reads planes q-1
-//    (rows r-1..r+1) and q-2 (row r) there, and u^{n+1}(q) is the thread's own
-//    step-(n+1) result; one CTA barrier per plane orders the ring and the TMA
-//    refills (a warp's only read of the oldest slot is its own row).
-template <typename T, int TY> struct TbUGeom {
-    using B = TbGeom<T, TY, 4, 4>;  // box shapes (the plan's tensor maps)
-    static constexpr int VEC = B::VEC, TX = B::TX, TXO = B::TXO, UROW = B::UROW, UR = B::UR, PR = B::PR;
-    static constexpr int KROW = B::KROW, U_BYTES = B::U_BYTES, P_BYTES = B::P_BYTES, K_BYTES = B::K_BYTES;
-    static constexpr int U1_BYTES = B::U1_BYTES, U_TX = B::U_TX, PK_TX = B::PK_TX;
-    static constexpr int SU = 4, SP = 4, S1 = 3;
-    static constexpr int NW = TY + 2, NT = 32 * NW;
-    static constexpr int SMEM = SU * U_BYTES + SP * (P_BYTES + K_BYTES) + S1 * U1_BYTES + (SU + SP) * 8 + 128;
-};
-
-template <typename T, int TY, bool DYN, bool NM = false>
-__global__ void __launch_bounds__(TbUGeom<T, TY>::NT, 1)
-    k_volume2u(const __grid_constant__ CUtensorMap umap, const __grid_constant__ CUtensorMap pmap,
-               const __grid_constant__ CUtensorMap kmap, T *__restrict__ out1, T *__restrict__ out2, Grid g, T l2,
-               int z_lo, int z_hi, int zchunk, int tiles_x, int tiles_y, unsigned int *work)
-{
-    using G = TbUGeom<T, TY>;
-    using KW = typename Vec16<T>::K;
-    constexpr int VEC = G::VEC, TX = G::TX, TXO = G::TXO, UROW = G::UROW, SU = G::SU, SP = G::SP;
-    constexpr int UE = G::U_BYTES / (int)sizeof(T), PE = G::P_BYTES / (int)sizeof(T), U1E = G::U1_BYTES / (int)sizeof(T);
-    extern __shared__ __align__(1024) unsigned char smem_raw[];
-    unsigned char *const base = smem_raw;
-    T *us = (T *)base;                                                  // SU u^n slots
-    T *ps = (T *)(base + SU * G::U_BYTES);                              // SP u^{n-1} slots
-    uint8_t *ks = base + SU * G::U_BYTES + SP * G::P_BYTES;             // SP K slots
-    T *u1s = (T *)(base + SU * G::U_BYTES + SP * (G::P_BYTES + G::K_BYTES));  // 3 u^{n+1} planes
-    uint64_t *bar = (uint64_t *)((unsigned char *)u1s + G::S1 * G::U1_BYTES);
-    int *const s_next = (int *)(bar + SU + SP);
-    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-    constexpr int ISSUER = 0;  // warp 0 (no step n+2 row), lane 0 issues the TMA loads
-
-    if (tid == 0) {
-        if (tb::smem_u32(smem_raw) & 127u) __trap();
-        for (int i = 0; i < SU + SP; i++) tb::mbar_init(&bar[i], 1);
-        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-    }
-    __syncthreads();
-    uint32_t uph = 0, pph = 0;
-    const uint64_t pol = tb::policy_store();
-
-    const int nz = z_hi - z_lo;
-    const int nchunks = (nz + zchunk - 1) / zchunk;
-    const int tiles = tiles_x * tiles_y;
-    const int units = nchunks * tiles;
-    const int r = warp - 1;                          // this warp's step row (-1 .. TY)
-    const bool core = r >= 0 && r < TY;              // also step n+2 (and stores)
-    const int col = VEC + lane * VEC;                // this lane's vector in a u^n smem row
-    const int hcol = lane == 0 ? VEC - 1 : VEC + TX;  // x halo of lanes 0 / 31 in a u^n smem row
-    int unit = blockIdx.x, next_unit = 0;
-    if constexpr (DYN) {
-        if (tid == 0) *s_next = (int)atomicAdd(work, 1u);
-        __syncthreads();
-        unit = *s_next;
-    }
-    while (unit < units) {
-        if constexpr (DYN) {
-            if (tid == 0) next_unit = (int)atomicAdd(work, 1u);
-        }
-        const int chunk = unit / tiles, t = unit % tiles;
-        const int ty = t / tiles_x, tx = t % tiles_x;
-        const int pa = 1 + z_lo + chunk * zchunk;
-        const int pb = min(1 + z_hi, pa + zchunk);
-        const int ox = tx * TXO, oy = ty * TY;
-        const int ux = g.xo + ox - 2 * VEC, uy = oy - 1;
-        const int px = g.xo + ox - VEC, py = oy;
-        const int kx = px + k_shift(g);
-        const int kd = kx & 15;
-        // u^n plane p in slot (p - pa + 2) & 3, u^{n-1}/K plane p in slot (p - pa + 1) & 3
-        auto issue_u = [&](int p, int s) {
-            tb::mbar_expect_tx(&bar[s], G::U_TX);
-            tb::tma_load_3d((unsigned char *)us + s * G::U_BYTES, &umap, &bar[s], ux, uy, p);
-        };
-        auto issue_pk = [&](int p, int s) {
-            tb::mbar_expect_tx(&bar[SU + s], G::PK_TX);
-            tb::tma_load_3d((unsigned char *)ps + s * G::P_BYTES, &pmap, &bar[SU + s], px, py, p);
-            tb::tma_load_3d(ks + s * G::K_BYTES, &kmap, &bar[SU + s], kx - kd, py, p);
-        };
-        auto wait_u = [&](int s) {
-            tb::mbar_wait(&bar[s], (uph >> s) & 1);
-            uph ^= 1u << s;
-        };
-        auto wait_pk = [&](int s) {
-            tb::mbar_wait(&bar[SU + s], (pph >> s) & 1);
-            pph ^= 1u << s;
-        };
-        __syncthreads();  // the previous unit is done with every slot
-        if (tid == ISSUER) {
-            asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-            for (int i = 0; i < SU && pa - 2 + i <= pb + 1; i++) issue_u(pa - 2 + i, i);
-            for (int i = 0; i < SP && pa - 1 + i <= pb; i++) issue_pk(pa - 1 + i, i);
-        }
-        // u^n(pa-2) at this thread's rows: the z-1 neighbours of the first plane
-        T cprev[VEC];
-        wait_u(0);
-        *(uint4 *)cprev = *(const uint4 *)(us + (r + 2) * UROW + col);
-        __syncthreads();  // slot 0 is free
-        if (tid == ISSUER) {
-            asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-            if (pa + 2 <= pb + 1) issue_u(pa + 2, 0);
-        }
-        wait_u(1);
-        KW km = 0;  // K of plane q-1 at this thread's core vector
-        const bool lane_core = lane >= 1 && lane <= 30;
-        const int xv = ox + (lane - 1) * VEC;
-        const bool st_ok = core && lane_core && xv < g.nx && oy + r < g.ny;
-        const int64_t roff = (int64_t)(oy + r + 1) * g.pitch + g.xo + xv;
-        int s1_c = 0, s1_m = 2, s1_mm = 1;  // u^{n+1} slots of planes q, q-1, q-2
-        for (int q0 = pa - 1; q0 <= pb; q0 += 4) {
-#pragma unroll
-            for (int j = 0; j < 4; j++) {
-                const int q = q0 + j;
-                if (q > pb) break;
-                constexpr int dummy = 0;
-                (void)dummy;
-                const int su_c = (j + 1) & 3, su_p = (j + 2) & 3, sp = j;
-                wait_u(su_p);
-                wait_pk(sp);
-                const T *uq = us + su_c * UE, *uqp = us + su_p * UE;
-                const T *pq = ps + sp * PE;
-                const uint8_t *kq = ks + sp * G::K_BYTES;
-                T *u1w = u1s + s1_c * U1E;
-                // step n+1 on plane q at step row rr: u^{n+1} to shared memory;
-                // zm (u^n(q-1) of the row) in, the centre vector out
-                auto step1 = [&](int rr, const T *zm, T *o1, T *cen) -> KW {
-                    const int sr = rr + 2;
-                    T ym[VEC], yp[VEC], zp[VEC], pv[VEC];
-                    *(uint4 *)cen = *(const uint4 *)(uq + sr * UROW + col);
-                    *(uint4 *)ym = *(const uint4 *)(uq + (sr - 1) * UROW + col);
-                    *(uint4 *)yp = *(const uint4 *)(uq + (sr + 1) * UROW + col);
-                    *(uint4 *)zp = *(const uint4 *)(uqp + sr * UROW + col);
-                    *(uint4 *)pv = *(const uint4 *)(pq + (rr + 1) * TX + lane * VEC);
-                    const KW kw = *(const KW *)(kq + (rr + 1) * G::KROW + kd + lane * VEC);
-                    const T halo = uq[sr * UROW + hcol];
-                    T left = __shfl_up_sync(0xffffffffu, cen[VEC - 1], 1);
-                    T right = __shfl_down_sync(0xffffffffu, cen[0], 1);
-                    left = lane == 0 ? halo : left;
-                    right = lane == 31 ? halo : right;
-                    if constexpr (NM) {  // diagnostic: same traffic, one add per voxel (not exact)
-#pragma unroll
-                        for (int i = 0; i < VEC; i++) o1[i] = cen[i] + pv[i] + (left + right) + ym[i] + yp[i] + zm[i] + zp[i] + (T)(kw & 1);
-                    } else {
-                        vol_vec<T>(cen, ym, yp, zm, zp, pv, left, right, (uint32_t)kw, l2, o1);
-                    }
-                    *(uint4 *)(u1w + (rr + 1) * TX + lane * VEC) = *(const uint4 *)o1;
-                    return kw;
-                };
-                T o1[VEC], cc[VEC];
-                const KW kc = step1(r, cprev, o1, cc);
-                if (q >= pa && q < pb && st_ok)
-                    tb::st_v4_hint(out1 + (int64_t)q * g.plane + roff, *(const uint4 *)o1, pol);
-                // step n+2 on plane q-1, row r: u^{n+1}(q-1) rows r-1..r+1 and
-                // u^{n+1}(q-2) row r from shared memory, u^{n+1}(q) = o1,
-                // u^n(q-1) = cprev
-                if (core && q - 1 >= pa) {
-                    const T *u1r = u1s + s1_m * U1E, *u1rr = u1s + s1_mm * U1E;
-                    T c[VEC], ym[VEC], yp[VEC], zm[VEC], o2[VEC];
-                    *(uint4 *)c = *(const uint4 *)(u1r + (r + 1) * TX + lane * VEC);
-                    *(uint4 *)ym = *(const uint4 *)(u1r + r * TX + lane * VEC);
-                    *(uint4 *)yp = *(const uint4 *)(u1r + (r + 2) * TX + lane * VEC);
-                    *(uint4 *)zm = *(const uint4 *)(u1rr + (r + 1) * TX + lane * VEC);
-                    const T left = __shfl_up_sync(0xffffffffu, c[VEC - 1], 1);
-                    const T right = __shfl_down_sync(0xffffffffu, c[0], 1);
-                    if constexpr (NM) {
-#pragma unroll
-                        for (int i = 0; i < VEC; i++) o2[i] = c[i] + ym[i] + yp[i] + zm[i] + o1[i] + cprev[i] + (left + right) + (T)(km & 1);
-                    } else {
-                        vol_vec<T>(c, ym, yp, zm, o1, cprev, left, right, (uint32_t)km, l2, o2);
-                    }
-                    if (st_ok) tb::st_v4_hint(out2 + (int64_t)(q - 1) * g.plane + roff, *(const uint4 *)o2, pol);
-                }
-                km = kc;
-#pragma unroll
-                for (int i = 0; i < VEC; i++) cprev[i] = cc[i];
-                __syncthreads();  // u^n(q), u^{n-1}/K(q), u^{n+1}(q-2) no longer read
-                if (tid == ISSUER) {
-                    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-                    if (q + 4 <= pb + 1) issue_u(q + 4, su_c);
-                    if (q + 4 <= pb) issue_pk(q + 4, sp);
-                }
-                const int t1 = s1_mm;
-                s1_mm = s1_m;
-                s1_m = s1_c;
-                s1_c = t1;
-            }
-        }
-        if constexpr (DYN) {
-            if (tid == 0) *s_next = next_unit;
-            __syncthreads();
-            unit = *s_next;
-        } else {
-            unit += gridDim.x;
-        }
-    }
-    if (DYN && tid == 0) {
-        __threadfence();
-        if (atomicAdd(work + 1, 1u) == gridDim.x - 1) {
             atomicExch(work, 0u);
             atomicExch(work + 1, 0u);
         }
@@ -1075,23 +565,10 @@ static bool tb_map(CUtensorMap *m, CUtensorMapDataType dt, size_t esize, void *b
 }
 
 static constexpr int kTbTY = 32, kTbSU = 4, kTbSP = 4;
-// k_volume2u tile rows (RAFD_TBU_TY: 30, 26 or 22; TY + 2 warps per CTA)
-static int tbu_ty_env()
-{
-    static int v = -1;
-    if (v < 0) {
-        const char *e = getenv("RAFD_TBU_TY");
-        v = e ? atoi(e) : 30;
-        if (v != 30 && v != 26 && v != 22) v = 30;
-    }
-    return v;
-}
 
 struct TwoStepPlan {
     CUtensorMap umap[4], pmap[4], kmap;
     int tiles_x, tiles_y, grid, smem;
-    int kernel = 0;  // 0: k_volume2 (two rows per warp), 1..4: k_volume2w, 5: k_volume2u
-    int ty = 32;     // tile rows
     void *list = nullptr;  // shell positions (uint32 or int64), ascending
     uint8_t *nmask = nullptr;  // per shell entry: inside face neighbours (bits x-1, x+1, y-1, y+1, z-1, z+1)
     int64_t *wbase = nullptr;  // [n/32 + 1] boundary nodes before each 32-entry group of the list
@@ -1117,17 +594,6 @@ static int tb_dynamic_env()
     }
     return v;
 }
-// two-step volume kernel (RAFD_TB_KERNEL = 0: k_volume2; 1..4: k_volume2w
-// variant V = value - 1, bit 0 split barrier, bit 1 running store pointers)
-static int tb_kernel_env()
-{
-    static int v = -2;
-    if (v == -2) {
-        const char *e = getenv("RAFD_TB_KERNEL");
-        v = e ? atoi(e) : 0;
-    }
-    return v;
-}
 static constexpr int kTbDynMinChunk = 24;  // unset: dynamic for units of >= 24 planes (small rooms stay static)
 
 template <typename T>
@@ -1136,83 +602,29 @@ cudaError_t twostep_plan_create(const Grid &g, void *const u[4], uint8_t *K_allo
 {
     using G = TbGeom<T, kTbTY, kTbSU, kTbSP>;
     auto *pl = new TwoStepPlan();
-    {
-        const int kv = tb_kernel_env();
-        pl->kernel = kv >= 1 && kv <= 6 ? kv : 0;
-    }
-    // tile rows: 32 (k_volume2, k_volume2w), 30 (k_volume2u: 32 step-(n+1) rows, one per warp)
-    {
-        const char *e = getenv("RAFD_TB_STPOL");
-        const int v = e ? atoi(e) : 0;
-        cudaMemcpyToSymbol(tb::c_tb_stpol, &v, sizeof v);
-    }
-    const int TYp = pl->kernel >= 5 ? tbu_ty_env() : kTbTY;
-    pl->ty = TYp;
     const CUtensorMapDataType dt = sizeof(T) == 4 ? CU_TENSOR_MAP_DATA_TYPE_FLOAT32 : CU_TENSOR_MAP_DATA_TYPE_FLOAT64;
     bool ok = true;
     for (int k = 0; k < 4; k++) {
-        ok = ok && tb_map(&pl->umap[k], dt, sizeof(T), u[k], g, G::UROW, TYp + 4);
-        ok = ok && tb_map(&pl->pmap[k], dt, sizeof(T), u[k], g, G::TX, TYp + 2);
+        ok = ok && tb_map(&pl->umap[k], dt, sizeof(T), u[k], g, G::UROW, G::UR);
+        ok = ok && tb_map(&pl->pmap[k], dt, sizeof(T), u[k], g, G::TX, G::PR);
     }
-    ok = ok && tb_map(&pl->kmap, CU_TENSOR_MAP_DATA_TYPE_UINT8, 1, K_alloc, g, G::KROW, TYp + 2, k_shift(g));
+    ok = ok && tb_map(&pl->kmap, CU_TENSOR_MAP_DATA_TYPE_UINT8, 1, K_alloc, g, G::KROW, G::PR, k_shift(g));
     if (!ok) {
         delete pl;
         return cudaErrorNotSupported;
     }
     pl->tiles_x = (g.nx + G::TXO - 1) / G::TXO;
-    pl->tiles_y = (g.ny + TYp - 1) / TYp;
+    pl->tiles_y = (g.ny + kTbTY - 1) / kTbTY;
+    pl->smem = G::SMEM;
     pl->idx64 = idx64;
-    cudaError_t e = cudaSuccess;
+    auto kern = k_volume2<T, kTbTY, kTbSU, kTbSP, false>;
+    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, pl->smem);
+    if (e == cudaSuccess)
+        e = cudaFuncSetAttribute(k_volume2<T, kTbTY, kTbSU, kTbSP, true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                 pl->smem);
     int occ = 0;
-    if (pl->kernel == 0) {
-        pl->smem = G::SMEM;
-        auto kern = k_volume2<T, kTbTY, kTbSU, kTbSP, false>;
-        e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, pl->smem);
-        if (e == cudaSuccess)
-            e = cudaFuncSetAttribute(k_volume2<T, kTbTY, kTbSU, kTbSP, true>,
-                                     cudaFuncAttributeMaxDynamicSharedMemorySize, pl->smem);
-        if (e == cudaSuccess) e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kern, G::NT, pl->smem);
-    } else if (pl->kernel >= 5) {
-        auto setup = [&](auto tyc) {
-            constexpr int TYc = decltype(tyc)::value;
-            using W = TbUGeom<T, TYc>;
-            pl->smem = W::SMEM;
-            cudaError_t err = cudaFuncSetAttribute(k_volume2u<T, TYc, false>,
-                                                   cudaFuncAttributeMaxDynamicSharedMemorySize, pl->smem);
-            if (err == cudaSuccess)
-                err = cudaFuncSetAttribute(k_volume2u<T, TYc, true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                           pl->smem);
-            if (err == cudaSuccess)
-                err = cudaFuncSetAttribute(k_volume2u<T, TYc, true, true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                           pl->smem);
-            if (err == cudaSuccess)
-                err = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_volume2u<T, TYc, false>, W::NT,
-                                                                    pl->smem);
-            return err;
-        };
-        e = TYp == 22 ? setup(std::integral_constant<int, 22>())
-            : TYp == 26 ? setup(std::integral_constant<int, 26>())
-                        : setup(std::integral_constant<int, 30>());
-    } else {
-        using W = TbRowGeom<T, kTbTY>;
-        pl->smem = W::SMEM;
-        const void *kd = nullptr, *kdd = nullptr;
-        switch (pl->kernel - 1) {
-#define RAFD_W(v)                                          \
-    case v:                                                \
-        kd = (const void *)k_volume2w<T, kTbTY, false, v>; \
-        kdd = (const void *)k_volume2w<T, kTbTY, true, v>; \
-        break;
-            RAFD_W(0)
-            RAFD_W(1)
-            RAFD_W(2)
-            RAFD_W(3)
-#undef RAFD_W
-        }
-        e = cudaFuncSetAttribute(kd, cudaFuncAttributeMaxDynamicSharedMemorySize, pl->smem);
-        if (e == cudaSuccess) e = cudaFuncSetAttribute(kdd, cudaFuncAttributeMaxDynamicSharedMemorySize, pl->smem);
-        if (e == cudaSuccess) e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kd, W::NT, pl->smem);
-    }
+    if (e == cudaSuccess) e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kern, G::NT, pl->smem);
+    if (e == cudaSuccess && occ < 1) e = cudaErrorInvalidConfiguration;
     pl->grid = nsm * std::max(occ, 1);
     // the shell list
     const int64_t rows = (int64_t)g.lnz * g.ny;
@@ -1351,55 +763,7 @@ cudaError_t launch_volume2(const void *plan, const Grid &g, int cur_buf, int pre
     const long units = (long)tiles * ((z_hi - z_lo + zc - 1) / zc);
     const int grid = (int)std::min<long>(pl->grid, units);
     const int env = tb_dynamic_env();
-    const bool dyn = env == 1 || (env < 0 && zc >= kTbDynMinChunk);
-    if (pl->kernel >= 5) {
-        auto run = [&](auto tyc) {
-            constexpr int TYc = decltype(tyc)::value;
-            using W = TbUGeom<T, TYc>;
-            if (pl->kernel == 6)
-                k_volume2u<T, TYc, true, true><<<grid, W::NT, pl->smem, s>>>(pl->umap[cur_buf], pl->pmap[prev_buf],
-                                                                             pl->kmap, out1, out2, g, l2, z_lo, z_hi,
-                                                                             zc, pl->tiles_x, pl->tiles_y, pl->work);
-            else if (dyn)
-                k_volume2u<T, TYc, true><<<grid, W::NT, pl->smem, s>>>(pl->umap[cur_buf], pl->pmap[prev_buf],
-                                                                       pl->kmap, out1, out2, g, l2, z_lo, z_hi, zc,
-                                                                       pl->tiles_x, pl->tiles_y, pl->work);
-            else
-                k_volume2u<T, TYc, false><<<grid, W::NT, pl->smem, s>>>(pl->umap[cur_buf], pl->pmap[prev_buf],
-                                                                        pl->kmap, out1, out2, g, l2, z_lo, z_hi, zc,
-                                                                        pl->tiles_x, pl->tiles_y, nullptr);
-        };
-        if (pl->ty == 22)
-            run(std::integral_constant<int, 22>());
-        else if (pl->ty == 26)
-            run(std::integral_constant<int, 26>());
-        else
-            run(std::integral_constant<int, 30>());
-        return cudaGetLastError();
-    }
-    if (pl->kernel >= 1) {
-        using W = TbRowGeom<T, kTbTY>;
-#define RAFD_W(v)                                                                                                   \
-    case v:                                                                                                         \
-        if (dyn)                                                                                                    \
-            k_volume2w<T, kTbTY, true, v><<<grid, W::NT, pl->smem, s>>>(pl->umap[cur_buf], pl->pmap[prev_buf],     \
-                                                                        pl->kmap, out1, out2, g, l2, z_lo, z_hi, zc, \
-                                                                        pl->tiles_x, pl->tiles_y, pl->work);         \
-        else                                                                                                        \
-            k_volume2w<T, kTbTY, false, v><<<grid, W::NT, pl->smem, s>>>(pl->umap[cur_buf], pl->pmap[prev_buf],    \
-                                                                         pl->kmap, out1, out2, g, l2, z_lo, z_hi,   \
-                                                                         zc, pl->tiles_x, pl->tiles_y, nullptr);    \
-        break;
-        switch (pl->kernel - 1) {
-            RAFD_W(0)
-            RAFD_W(1)
-            RAFD_W(2)
-            RAFD_W(3)
-        }
-#undef RAFD_W
-        return cudaGetLastError();
-    }
-    if (dyn)
+    if (env == 1 || (env < 0 && zc >= kTbDynMinChunk))
         k_volume2<T, kTbTY, kTbSU, kTbSP, true><<<grid, G::NT, pl->smem, s>>>(
             pl->umap[cur_buf], pl->pmap[prev_buf], pl->kmap, out1, out2, g, l2, z_lo, z_hi, zc, pl->tiles_x,
             pl->tiles_y, pl->work);
