@@ -7,7 +7,8 @@ a2-a6; the once-per-room classification a1 is timed inside `e2e`).  Workload at
 N=1: BASELINE.json configs[3], the C4 hall 1536x1024x704 (1.107e9 voxels), box,
 FD-MM with 3 branches and 8 materials, fp32; the line also carries
 `single_step` (the same room at one step per sweep: Listings 2-4 iterated) and
-`strong_t1` (C5, configs[4], on one GPU: T_1 of the strong-scaling curve).
+`strong_t1` (C5, configs[4], on one GPU: T_1 of the strong-scaling curve) and
+`fp64` (the C4 room in double precision: the metric is quoted for fp32 and fp64).
 N>1 (torchrun, one rank per GPU): C5 2048x1536x2560 (8.05e9 voxels) split into N
 z-slabs (rafd_slab_plan; strong scaling, E_p = T_1 / (p T_p)), one-plane halo
 exchange per step (NCCL send/recv by default), then a bitwise parity check of
@@ -442,6 +443,17 @@ def run_rafd(args, rank, world, local_rank):
         rafd.rafd_release_cached_memory(local_rank)
         torch.cuda.synchronize()
         torch.cuda.empty_cache()
+        # the metric is "Gvoxel-updates/s (fp32/fp64)": the same C4 room in fp64
+        if prec == 32:
+            r6, tb6, _, _ = make_room(cfg, 64, 0, 1, local_rank, args.transport, stream, args.tb)
+            rec6 = sub_record(r6, args.steps, args.warmup, stream, 64, tb6, peak)
+            rec6["workload"] = "C4: 1536x1024x704 box room, FD-MM MB=3 M=8, fp64, 1 GPU"
+            out["fp64"] = rec6
+            r6.destroy()
+            del r6
+            rafd.rafd_release_cached_memory(local_rank)
+            torch.cuda.synchronize()
+            torch.cuda.empty_cache()
     e2e = run_e2e(args, cfg, prec, *I.config_materials(cfg), rank, world, local_rank, plan,
                   world > 1 and args.transport == "nccl")
     if rank == 0:
@@ -769,7 +781,7 @@ def main():
     ap.add_argument("--precision", type=int, default=None)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-sub-records", action="store_true",
-                    help="N=1: skip the single_step (C4, one step per sweep) and strong_t1 (C5 on one GPU) records")
+                    help="N=1: skip the single_step (C4, one step per sweep), strong_t1 (C5 on one GPU) and fp64 (C4) records")
     ap.add_argument("--tb", type=int, default=0, choices=[0, 1, 2],
                     help="steps per HBM sweep (2: temporal blocking); 0 = auto: 2 for rooms of >= 2^25 "
                          "voxels per GPU, 1 below (measured: C2 256^3 is faster with single steps, C3 and "
