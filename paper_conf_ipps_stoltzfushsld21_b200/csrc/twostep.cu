@@ -490,7 +490,9 @@ __global__ void __launch_bounds__(256)
             const T xm = (m & 1) ? u1[p - 1] : (T)0, xp = (m & 2) ? u1[p + 1] : (T)0;
             const T ym = (m & 4) ? u1[p - g.pitch] : (T)0, yp = (m & 8) ? u1[p + g.pitch] : (T)0;
             const T zm = (m & 16) ? u1[p - g.plane] : (T)0, zp = (m & 32) ? u1[p + g.plane] : (T)0;
-            const T c = u1[p], pv = u0[p];
+            // at a node u^n is its u_b slot (loaded above as uprev, the same value the
+            // boundary update uses): the grid copy is read only at the other entries
+            const T c = u1[p], pv = node ? uprev : u0[p];
             T s = R::add(xm, xp);
             s = R::add(s, ym);
             s = R::add(s, yp);
