@@ -49,6 +49,35 @@ struct PhaseTrace {
     }
 };
 
+// Work enqueued on a side stream while the main stream does something else
+// (setup only): the destructor makes the main stream wait for it, so every
+// later use -- and every error path, which synchronises the main stream before
+// freeing -- is ordered after it.
+struct SideWork {
+    cudaStream_t main, side;
+    cudaEvent_t ev = nullptr;
+    SideWork(cudaStream_t m, cudaStream_t sd) : main(m), side(sd) {}
+    void done()
+    {
+        if (ev) return;
+        if (cudaEventCreateWithFlags(&ev, cudaEventDisableTiming) != cudaSuccess || cudaEventRecord(ev, side) != cudaSuccess) {
+            cudaStreamSynchronize(side);  // fall back to a host wait
+            if (ev) cudaEventDestroy(ev);
+            ev = nullptr;
+            return;
+        }
+    }
+    ~SideWork()
+    {
+        if (ev) {
+            cudaStreamWaitEvent(main, ev, 0);
+            cudaEventDestroy(ev);
+        } else {
+            cudaStreamSynchronize(side);  // an error path left before done()
+        }
+    }
+};
+
 static int set_err(int code, const char *fmt, ...)
 {
     char buf[512];
@@ -349,8 +378,13 @@ template <typename T> static int create_t(rafd_room *r, const rafd_room_desc *d)
         if ((rc = dmalloc(r, &r->u[k], (size_t)g.total * sizeof(T) + 64))) return rc;
     tr.mark(r->stream, "alloc K, u[2]");
     CK(cudaMemsetAsync(r->K_alloc, 0, (size_t)g.total + 64, r->stream));
-    for (int k = 0; k < 2; k++) CK(cudaMemsetAsync(r->u[k], 0, (size_t)g.total * sizeof(T) + 64, r->stream));
-    tr.mark(r->stream, "memset K, u[2]");
+    // the two field buffers are zeroed on the side stream while the mask streams
+    // in over PCIe (C4: 1.5 ms of memset hidden behind the 20 ms H2D); the main
+    // stream waits for it when create_t returns
+    SideWork zero_u(r->stream, r->cap_stream);
+    for (int k = 0; k < 2; k++) CK(cudaMemsetAsync(r->u[k], 0, (size_t)g.total * sizeof(T) + 64, r->cap_stream));
+    zero_u.done();
+    tr.mark(r->stream, "memset K");
 
     // ---- classification (row a1)
     // the mask is streamed in full (DMA staging beats zero-copy reads for it);
@@ -470,10 +504,11 @@ template <typename T> static int create_t(rafd_room *r, const rafd_room_desc *d)
     const char *env = getenv("RAFD_VOLUME_KERNEL");
     if (!(env && strcmp(env, "v0") == 0)) {
         CK(volume_plan_create<T>(g, r->u, r->K_alloc, r->nsm, &r->vplan));
+        tr.mark(r->stream, "volume plan: maps, attributes");
         const char *sk = getenv("RAFD_SKIP_EMPTY");  // skipping of all-outside tile-planes (default on)
         if (!(sk && strcmp(sk, "0") == 0)) CK(volume_plan_occupancy(r->vplan, g, r->K, r->stream));
     }
-    tr.mark(r->stream, "volume plan");
+    tr.mark(r->stream, "volume plan: occupancy");
     // boundary update fused into the volume kernel with RAFD_FUSED=1 (DESIGN.md
     // §6; needs the default tiling, MB <= 4, Nb < 2^31).  Off by default: the
     // first fused form is latency-bound at x-wall rows (5.6 ms vs 2.55 ms).
@@ -1660,22 +1695,27 @@ template <typename T> static int enable_twostep_t(rafd_room *r)
             }
     };
     PhaseTrace tr("rafd_set_temporal_blocking(2)");
-    for (int k = 2; k < 4 && rc == RAFD_OK; k++)
-        if (!nu[k]) {
-            if ((rc = dmalloc(r, &nu[k], fb)) == RAFD_OK) {
-                fresh[k] = true;
-                e = cudaMemsetAsync(nu[k], 0, fb, r->stream);
-                if (e != cudaSuccess) rc = -1;
+    {
+        // the second pair is zeroed on the side stream while the plans are built
+        SideWork zero_u(r->stream, r->cap_stream);
+        for (int k = 2; k < 4 && rc == RAFD_OK; k++)
+            if (!nu[k]) {
+                if ((rc = dmalloc(r, &nu[k], fb)) == RAFD_OK) {
+                    fresh[k] = true;
+                    e = cudaMemsetAsync(nu[k], 0, fb, r->cap_stream);
+                    if (e != cudaSuccess) rc = -1;
+                }
             }
-        }
-    tr.mark(r->stream, "alloc + memset u[2..3]");
-    // the single-step kernel needs TMA maps of the second pair too
-    if (rc == RAFD_OK && e == cudaSuccess) e = volume_plan_create<T>(r->g, nu, r->K_alloc, r->nsm, &vp);
-    // (the occupancy table is taken over from the current plan at the commit below)
-    tr.mark(r->stream, "volume plan");
-    if (rc == RAFD_OK && e == cudaSuccess)
-        e = twostep_plan_create<T>(r->g, nu, r->K_alloc, r->K, r->idx64, r->nsm, r->stream, &tp, &nsh);
-    tr.mark(r->stream, "two-step plan + shell list");
+        zero_u.done();
+        tr.mark(r->stream, "alloc u[2..3]");
+        // the single-step kernel needs TMA maps of the second pair too
+        if (rc == RAFD_OK && e == cudaSuccess) e = volume_plan_create<T>(r->g, nu, r->K_alloc, r->nsm, &vp);
+        // (the occupancy table is taken over from the current plan at the commit below)
+        tr.mark(r->stream, "volume plan");
+        if (rc == RAFD_OK && e == cudaSuccess)
+            e = twostep_plan_create<T>(r->g, nu, r->K_alloc, r->K, r->idx64, r->nsm, r->stream, &tp, &nsh);
+        tr.mark(r->stream, "two-step plan + shell list");
+    }  // the main stream waits for the zeroing here (before any use, synchronisation or undo)
     Ctl<T> c;
     if (rc == RAFD_OK && e == cudaSuccess) {
         if ((rc = pull_ctl<T>(r, c)) == RAFD_OK) e = twostep_set_source(tp, c.src_pos, r->g);
