@@ -341,6 +341,40 @@ cudaError_t launch_scatter_mask(const Grid &g, const uint8_t *mask_chunk, int zp
     return cudaGetLastError();
 }
 
+// Bit-packed chunk (maskpack.cu): nzc planes from local padded plane zp0, rows
+// of rw 32-bit words, bit i of word w = voxel x = 32 w + i.  One thread per
+// word writes the 32 K bytes it covers (0x80 where set, as k_scatter_mask).
+__global__ void k_scatter_mask_bits(Grid g, const uint32_t *__restrict__ bits, int rw, int zp0, int nzc,
+                                    uint8_t *__restrict__ K)
+{
+    const int64_t nw = (int64_t)nzc * g.ny * rw;
+    for (int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; t < nw; t += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t row = t / rw;
+        const int wi = (int)(t - row * rw), x0 = 32 * wi;
+        const int64_t y = row % g.ny, z = row / g.ny;
+        const uint32_t b = bits[t];
+        uint8_t *k = K + pidx(g, zp0 + z, y, x0);
+        if (x0 + 32 <= g.nx) {  // x = 0 of a K row is 16-byte aligned, x0 a multiple of 32
+            uint32_t e[8];
+#pragma unroll
+            for (int j = 0; j < 8; j++) e[j] = ((((b >> (4 * j)) & 15u) * 0x00204081u) & 0x01010101u) * 0x80u;
+            *(uint4 *)k = make_uint4(e[0], e[1], e[2], e[3]);
+            *(uint4 *)(k + 16) = make_uint4(e[4], e[5], e[6], e[7]);
+        } else {
+            for (int i = 0; i < g.nx - x0; i++) k[i] = ((b >> i) & 1u) ? 0x80 : 0;
+        }
+    }
+}
+
+cudaError_t launch_scatter_mask_bits(const Grid &g, const uint32_t *bits, int rw, int zp0, int nzc, uint8_t *K,
+                                     cudaStream_t s)
+{
+    const int64_t nw = (int64_t)nzc * g.ny * rw;
+    if (nw == 0) return cudaSuccess;
+    k_scatter_mask_bits<<<grid_for(nw, 256), 256, 0, s>>>(g, bits, rw, zp0, nzc, K);
+    return cudaGetLastError();
+}
+
 cudaError_t launch_count_k(const Grid &g, uint8_t *K, cudaStream_t s)
 {
     const int64_t items = (int64_t)g.lnz * g.ny * ((g.nx + 15) / 16);

@@ -158,6 +158,11 @@ cudaError_t launch_find_node(const void *bpos, bool idx64, int64_t Nb, int64_t p
 // classification: flags -> K (in place, bit 7 trick), counts, compaction
 cudaError_t launch_scatter_mask(const Grid &g, const uint8_t *mask_chunk, int zp0, int nzc,
                                 uint8_t *K, cudaStream_t s);
+cudaError_t launch_scatter_mask_bits(const Grid &g, const uint32_t *bits, int rw, int zp0, int nzc, uint8_t *K,
+                                     cudaStream_t s);
+// host side of the bit-packed mask upload (maskpack.cu)
+int pack_threads();
+void pack_mask_rows(const uint8_t *mask, int64_t nrows, int nx, uint32_t *out, int rw, int nthreads);
 cudaError_t launch_count_k(const Grid &g, uint8_t *K, cudaStream_t s);
 cudaError_t launch_finish_k(const Grid &g, uint8_t *K, unsigned long long *hist8,
                             cudaStream_t s);

@@ -14,6 +14,10 @@
 #include <stdarg.h>
 #include <stdio.h>
 #include <stdlib.h>
+
+#include <mutex>
+#include <thread>
+#include <vector>
 #include <string.h>
 
 #include <algorithm>
@@ -353,6 +357,90 @@ static int for_plane_chunks(rafd_room *r, const void *src, int src_z0, bool dev,
 
 static const size_t kStagingBytes = 256ull << 20;
 
+// Bit-packed upload of a host mask (maskpack.cu, classify.cu k_scatter_mask_bits):
+// the classification needs one bit per voxel, the mask has a byte (C4: the
+// 1.1 GB byte mask crossed PCIe in 20.4 ms).  Host threads each pack a range of
+// planes into a pinned buffer and issue its copy as soon as it is packed, so the
+// 1/8-size copies overlap the packing; the device expands the bits into K.
+// Rounds of at most kStagingBytes packed.  The pinned buffer is shared by the
+// process's rooms (grown on demand).  RAFD_MASK_BITS=0 keeps the byte stream.
+// Returns -1 when not applicable (the caller then streams bytes).
+static std::mutex g_pack_mu;
+static void *g_pack_host = nullptr;
+static size_t g_pack_bytes = 0;
+
+static int upload_mask_bits(rafd_room *r, const uint8_t *mask, int mz0, int zg0, int nplanes, void *staging)
+{
+    if (const char *e = getenv("RAFD_MASK_BITS"))
+        if (atoi(e) == 0) return -1;
+    const Grid &g = r->g;
+    const int rw = (r->nx + 31) / 32;
+    const size_t plane_b = (size_t)r->ny * rw * 4, nxny = (size_t)r->nx * r->ny;
+    if (nplanes <= 0 || plane_b > kStagingBytes) return -1;
+    const int per_round = (int)std::min<size_t>((size_t)nplanes, kStagingBytes / plane_b);
+    std::lock_guard<std::mutex> lk(g_pack_mu);
+    const size_t need = (size_t)per_round * plane_b;
+    if (g_pack_bytes < need) {
+        if (g_pack_host) cudaFreeHost(g_pack_host);
+        g_pack_host = nullptr;
+        g_pack_bytes = 0;
+        if (cudaHostAlloc(&g_pack_host, need, cudaHostAllocPortable) != cudaSuccess) {
+            cudaGetLastError();
+            g_pack_host = nullptr;
+            return -1;
+        }
+        g_pack_bytes = need;
+    }
+    const int nt = std::max(1, std::min(pack_threads(), per_round));
+    std::vector<cudaStream_t> cs(nt, nullptr);
+    std::vector<cudaEvent_t> ce(nt, nullptr);
+    cudaError_t e = cudaSuccess;
+    for (int t = 0; t < nt && e == cudaSuccess; t++) {
+        e = cudaStreamCreateWithFlags(&cs[t], cudaStreamNonBlocking);
+        if (e == cudaSuccess) e = cudaEventCreateWithFlags(&ce[t], cudaEventDisableTiming);
+    }
+    for (int z = zg0; z < zg0 + nplanes && e == cudaSuccess; z += per_round) {
+        const int n = std::min(per_round, zg0 + nplanes - z);
+        // the previous round's expansion has read the device buffer (stream order
+        // on r->stream is not enough: the copies run on the packing threads' streams)
+        e = cudaStreamSynchronize(r->stream);
+        if (e != cudaSuccess) break;
+        std::vector<cudaError_t> te(nt, cudaSuccess);
+        std::vector<std::thread> th;
+        th.reserve(nt);
+        for (int t = 0; t < nt; t++) {
+            const int p0 = (int)((int64_t)n * t / nt), p1 = (int)((int64_t)n * (t + 1) / nt);
+            if (p0 >= p1) continue;
+            th.emplace_back([&, t, p0, p1] {
+                cudaSetDevice(r->device);  // a new thread starts on device 0
+                uint32_t *hb = (uint32_t *)((char *)g_pack_host + (size_t)p0 * plane_b);
+                pack_mask_rows(mask + (size_t)(z + p0 - mz0) * nxny, (int64_t)(p1 - p0) * r->ny, r->nx, hb, rw, 1);
+                te[t] = cudaMemcpyAsync((char *)staging + (size_t)p0 * plane_b, hb, (size_t)(p1 - p0) * plane_b,
+                                        cudaMemcpyHostToDevice, cs[t]);
+                if (te[t] == cudaSuccess) te[t] = cudaEventRecord(ce[t], cs[t]);
+            });
+        }
+        for (auto &t : th) t.join();
+        for (int t = 0; t < nt && e == cudaSuccess; t++) {
+            const int p0 = (int)((int64_t)n * t / nt), p1 = (int)((int64_t)n * (t + 1) / nt);
+            if (p0 >= p1) continue;
+            e = te[t];
+            if (e == cudaSuccess) e = cudaStreamWaitEvent(r->stream, ce[t], 0);
+        }
+        if (e == cudaSuccess)
+            e = launch_scatter_mask_bits(g, (const uint32_t *)staging, rw, z - r->z0 + 1, n, r->K, r->stream);
+    }
+    // the pinned buffer is reused by the next room: drain before unlocking
+    const cudaError_t e2 = cudaStreamSynchronize(r->stream);
+    if (e == cudaSuccess) e = e2;
+    for (int t = 0; t < nt; t++) {
+        if (cs[t]) cudaStreamSynchronize(cs[t]), cudaStreamDestroy(cs[t]);
+        if (ce[t]) cudaEventDestroy(ce[t]);
+    }
+    if (e != cudaSuccess) return set_err(RAFD_E_CUDA, "mask upload: %s", cudaGetErrorString(e));
+    return RAFD_OK;
+}
+
 template <typename T> static int create_t(rafd_room *r, const rafd_room_desc *d)
 {
     const int64_t nxny = (int64_t)r->nx * r->ny;
@@ -396,11 +484,14 @@ template <typename T> static int create_t(rafd_room *r, const rafd_room_desc *d)
     if ((!mdev || (d->matmap && !matmap_dv)) && (rc = dmalloc(r, &staging, kStagingBytes))) return rc;
     const int zlo = std::max(0, r->z0 - 1), zhi = std::min(r->nz, r->z1 + 1);  // incl. ghost planes
     const int mz0 = d->mask_z0;
-    rc = for_plane_chunks(r, mdev ? mask_dv : d->mask, mz0, mdev, (size_t)nxny, zlo, zhi - zlo, staging, kStagingBytes,
-                          [&](const void *chunk, int zg, int n) -> int {
-                              CK(launch_scatter_mask(g, (const uint8_t *)chunk, zg - r->z0 + 1, n, r->K, r->stream));
-                              return RAFD_OK;
-                          });
+    rc = mdev ? -1 : upload_mask_bits(r, (const uint8_t *)d->mask, mz0, zlo, zhi - zlo, staging);
+    if (rc == -1)
+        rc = for_plane_chunks(r, mdev ? mask_dv : d->mask, mz0, mdev, (size_t)nxny, zlo, zhi - zlo, staging,
+                              kStagingBytes, [&](const void *chunk, int zg, int n) -> int {
+                                  CK(launch_scatter_mask(g, (const uint8_t *)chunk, zg - r->z0 + 1, n, r->K,
+                                                         r->stream));
+                                  return RAFD_OK;
+                              });
     if (rc) return rc;
     tr.mark(r->stream, "mask H2D + scatter");
     CK(launch_count_k(g, r->K, r->stream));
