@@ -662,6 +662,9 @@ def run_e2e(args, cfg, prec, beta0, D, E, F, rank, world, local_rank, plan, mult
             "h2d_bytes_per_step": int(h2d // steps), "d2h_bytes_per_step": int(d2h // steps),
             "wall_s": round(tmax, 3), "wall_s_runs": [round(w, 3) for w in walls],
             "cold_wall_s": round(walls[0], 3),
+            "h2d_bytes_note": "the input tensors handed to rafd_create (mask, matmap) and the source signal; "
+                              "the library moves the mask over PCIe bit-packed (host threads pack it: 1/8 of "
+                              "its bytes) and reads the matmap only at boundary nodes",
             "includes": "rafd_create from pinned host mask+matmap (H2D, device classification), "
                         "set_source/set_receivers, per step rafd_step(1)+rafd_read_receivers (D2H), destroy; "
                         "median of %d runs (the first allocates from the driver, later ones reuse the library's "
