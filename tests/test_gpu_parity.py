@@ -79,6 +79,37 @@ def test_classification_bit_exact(orc, room):
     check_classification(o, g)
 
 
+@pytest.mark.parametrize("dims", [(45, 37, 19), (64, 20, 9), (33, 1, 70), (300, 7, 5)])
+def test_mask_upload_bit_packed_and_byte_stream_agree(orc, dims, monkeypatch):
+    """A host mask crosses PCIe bit-packed (host threads, AVX2) unless
+    RAFD_MASK_BITS=0 streams its bytes: both give the oracle's classification,
+    for any nonzero byte as "inside", x extents that are not multiples of 32,
+    and a slab whose mask holds only its planes plus the two ghost planes."""
+    nx, ny, nz = dims
+    rng = np.random.default_rng(nx * 7 + ny)
+    mask = rng.choice(np.array([0, 1, 7, 255], np.uint8), size=(nz, ny, nx), p=[0.15, 0.65, 0.1, 0.1])
+    mm = I.material_map(torch.from_numpy((mask != 0).astype(np.uint8)), "random", 5).numpy()
+    o = orc.OracleRoom((mask != 0).astype(np.uint8), LAM, 32, [0.1] * 5, matmap=mm)
+    for bits in ("1", "0"):
+        monkeypatch.setenv("RAFD_MASK_BITS", bits)
+        g = rafd.Room(mask, LAM, 32, [0.1] * 5, matmap=mm)
+        check_classification(o, g)
+        g.destroy()
+    # a slab's planes [z0, z1) from a mask that starts at plane z0 - 1
+    z0, z1 = nz // 3, nz - nz // 3
+    if z1 - z0 >= 1 and z0 >= 1:
+        sub = np.ascontiguousarray(mask[z0 - 1:z1 + 1])
+        msub = np.ascontiguousarray(mm[z0 - 1:z1 + 1])
+        Ko = o.classification()[0]
+        for bits in ("1", "0"):
+            monkeypatch.setenv("RAFD_MASK_BITS", bits)
+            g = rafd.Room(sub, LAM, 32, [0.1] * 5, matmap=msub, rank=0, nranks=3, z_begin=z0, z_end=z1,
+                          mask_z0=z0 - 1, dims=(nx, ny, nz))
+            Kg = g.get_classification()[0]
+            assert np.array_equal(Kg, Ko[z0:z1]), bits
+            g.destroy()
+
+
 def test_classification_region_rule_and_device_inputs(orc):
     mask_t = I.dome_mask(64, 48, 40)
     mm_t = I.material_map(mask_t, "region", 8)
