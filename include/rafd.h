@@ -139,7 +139,12 @@ typedef struct rafd_kernel_times {
 /* Create a room: validates lambda / tables / dims, copies mask and matmap to
  * the device, classifies voxels on the device (K, ascending boundary list,
  * K_b, mat_b: PAPER.md:306-323, 390-393, 411-412), allocates and zeroes the
- * two field buffers, the boundary-node ring u_b and the branch state.  Errors: INVAL, UNSTABLE,
+ * two field buffers, the boundary-node ring u_b and the branch state.  A host
+ * mask is read by host threads (one per core, up to 32) that pack it to one
+ * bit per voxel in a process-wide pinned buffer before the copy (environment
+ * RAFD_MASK_BITS=0: copy the bytes); a host matmap is read in place at the
+ * boundary nodes (pinned) or streamed (pageable).  The inputs are only read,
+ * and not used after the call returns.  Errors: INVAL, UNSTABLE,
  * NONPASSIVE, MATERIAL, NOMEM, CUDA, NCCL.  *out is NULL on error. */
 int rafd_create(const rafd_room_desc *d, rafd_room **out);
 
@@ -288,8 +293,9 @@ int rafd_slab_plan(int32_t nx, int32_t ny, int32_t nz, const uint8_t *mask, int3
  * size reuses them.  This call frees every cached block of `device`, e.g.
  * before another library allocates large buffers (like
  * torch.cuda.empty_cache()).  Waits for the device.  Rooms still alive keep
- * their memory.  INVAL (device < 0), CUDA.  Environment RAFD_POOL=0 makes
- * rooms use cudaMalloc / cudaFree directly. */
+ * their memory.  Also frees the pinned host buffer of the bit-packed mask
+ * upload (rafd_create).  INVAL (device < 0), CUDA.  Environment RAFD_POOL=0
+ * makes rooms use cudaMalloc / cudaFree directly. */
 int rafd_release_cached_memory(int32_t device);
 
 /* 128-byte NCCL unique id for a multi-GPU room (call on rank 0, broadcast). */

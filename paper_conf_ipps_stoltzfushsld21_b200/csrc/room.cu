@@ -735,6 +735,12 @@ extern "C" int rafd_release_cached_memory(int32_t device)
     CK(cudaSetDevice(device));
     CK(cudaDeviceSynchronize());
     dev_cache_trim(device, 0);
+    {  // the pinned staging of the bit-packed mask upload (process-wide)
+        std::lock_guard<std::mutex> lk(g_pack_mu);
+        if (g_pack_host) cudaFreeHost(g_pack_host);
+        g_pack_host = nullptr;
+        g_pack_bytes = 0;
+    }
     return RAFD_OK;
 }
 
