@@ -406,20 +406,25 @@ static int upload_mask_bits(rafd_room *r, const uint8_t *mask, int mz0, int zg0,
         e = cudaStreamSynchronize(r->stream);
         if (e != cudaSuccess) break;
         std::vector<cudaError_t> te(nt, cudaSuccess);
+        auto part = [&](int t) {
+            const int p0 = (int)((int64_t)n * t / nt), p1 = (int)((int64_t)n * (t + 1) / nt);
+            if (p0 >= p1) return;
+            cudaSetDevice(r->device);  // a new thread starts on device 0
+            uint32_t *hb = (uint32_t *)((char *)g_pack_host + (size_t)p0 * plane_b);
+            pack_mask_rows(mask + (size_t)(z + p0 - mz0) * nxny, (int64_t)(p1 - p0) * r->ny, r->nx, hb, rw, 1);
+            te[t] = cudaMemcpyAsync((char *)staging + (size_t)p0 * plane_b, hb, (size_t)(p1 - p0) * plane_b,
+                                    cudaMemcpyHostToDevice, cs[t]);
+            if (te[t] == cudaSuccess) te[t] = cudaEventRecord(ce[t], cs[t]);
+        };
         std::vector<std::thread> th;
         th.reserve(nt);
-        for (int t = 0; t < nt; t++) {
-            const int p0 = (int)((int64_t)n * t / nt), p1 = (int)((int64_t)n * (t + 1) / nt);
-            if (p0 >= p1) continue;
-            th.emplace_back([&, t, p0, p1] {
-                cudaSetDevice(r->device);  // a new thread starts on device 0
-                uint32_t *hb = (uint32_t *)((char *)g_pack_host + (size_t)p0 * plane_b);
-                pack_mask_rows(mask + (size_t)(z + p0 - mz0) * nxny, (int64_t)(p1 - p0) * r->ny, r->nx, hb, rw, 1);
-                te[t] = cudaMemcpyAsync((char *)staging + (size_t)p0 * plane_b, hb, (size_t)(p1 - p0) * plane_b,
-                                        cudaMemcpyHostToDevice, cs[t]);
-                if (te[t] == cudaSuccess) te[t] = cudaEventRecord(ce[t], cs[t]);
-            });
+        int spawned = 0;
+        try {
+            for (int t = 1; t < nt; t++, spawned++) th.emplace_back(part, t);
+        } catch (...) {  // no threads to be had: the caller's thread packs the rest
         }
+        part(0);
+        for (int t = 1 + spawned; t < nt; t++) part(t);
         for (auto &t : th) t.join();
         for (int t = 0; t < nt && e == cudaSuccess; t++) {
             const int p0 = (int)((int64_t)n * t / nt), p1 = (int)((int64_t)n * (t + 1) / nt);
