@@ -392,6 +392,12 @@ def run_rafd(args, rank, world, local_rank):
                 "algorithmic_bytes_per_launch": vol_bytes,
                 "avg_launch_ms": round(launch_ms, 5), "launches_per_step": kt["volume_launches"] / args.steps,
                 "peak_source": peak_src,
+                **({"traffic_frac_of_peak": round(traffic / (launch_ms * 1e-3) / 1e9 / peak, 4),
+                    "note": "k_volume2 moves its ncu DRAM traffic (1.04x the algorithmic bytes: overlapped-tile "
+                            "re-reads) at traffic_frac_of_peak; capping the persistent grid shows it bound per SM "
+                            "(time = ceil(units / CTAs) x 0.19 ms for 100..148 CTAs), "
+                            "profiles/r02_volume2_alternatives_ab.txt"}
+                   if tb == 2 and world == 1 and traffic else {}),
             },
             "kernels": {
                 "volume_ms_per_step": round(vol_ms, 5), "boundary_ms_per_step": round(bnd_ms, 5),
