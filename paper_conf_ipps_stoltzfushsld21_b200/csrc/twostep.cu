@@ -290,10 +290,16 @@ __global__ void __launch_bounds__(TbGeom<T, TY, SU, SP>::NT, 1)
                 *(uint4 *)yp = *(const uint4 *)(uq + (sr + 1) * UROW + col);
                 *(uint4 *)pv = *(const uint4 *)(pq + (r + 1) * TX + lane * VEC);
                 kqv[k] = *(const KW *)(kq + (r + 1) * G::KROW + kd + lane * VEC);
+                // the x halo of lanes 0 / 31 into registers of their own, loaded
+                // before the shuffles (one load and one shuffle in flight together,
+                // not a shuffle, then a load into the same register)
+                T hl = (T)0, hr = (T)0;
+                if (lane == 0) hl = uq[sr * UROW + VEC - 1];
+                if (lane == 31) hr = uq[sr * UROW + VEC + TX];
                 T left = __shfl_up_sync(0xffffffffu, unc[k][VEC - 1], 1);
                 T right = __shfl_down_sync(0xffffffffu, unc[k][0], 1);
-                if (lane == 0) left = uq[sr * UROW + VEC - 1];
-                if (lane == 31) right = uq[sr * UROW + VEC + TX];
+                left = lane == 0 ? hl : left;
+                right = lane == 31 ? hr : right;
                 vol_vec<T>(unc[k], ym, yp, unm[k], unp[k], pv, left, right, (uint32_t)kqv[k], l2, o1p[k]);
                 *(uint4 *)(u1w + (r + 1) * TX + lane * VEC) = *(const uint4 *)o1p[k];
                 if (q >= pa && q < pb && r >= 0 && r < TY && x_ok && oy + r < g.ny) {
