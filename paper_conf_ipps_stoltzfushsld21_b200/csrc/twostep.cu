@@ -313,15 +313,17 @@ __global__ void __launch_bounds__(TbGeom<T, TY, SU, SP>::NT, 1)
                 const T *u1r = u1s + ((q - 1) & 1) * (G::U1_BYTES / (int)sizeof(T));
 #pragma unroll
                 for (int k = 0; k < 2; k++) {
-                    const int r = r0 + k;
-                    if (r < 0 || r >= TY) continue;  // warp-uniform
+                    // every warp runs both rows (uniform control flow, no divergent
+                    // shuffles); the halo rows -1 and TY of warps 0 and NW-1 read a
+                    // clamped row and are not stored
+                    const int r = r0 + k, rr = min(max(r, 0), TY - 1);
                     T ym[VEC], yp[VEC], o2[VEC];
-                    *(uint4 *)ym = *(const uint4 *)(u1r + r * TX + lane * VEC);
-                    *(uint4 *)yp = *(const uint4 *)(u1r + (r + 2) * TX + lane * VEC);
+                    *(uint4 *)ym = *(const uint4 *)(u1r + rr * TX + lane * VEC);
+                    *(uint4 *)yp = *(const uint4 *)(u1r + (rr + 2) * TX + lane * VEC);
                     const T left = __shfl_up_sync(0xffffffffu, o1c[k][VEC - 1], 1);
                     const T right = __shfl_down_sync(0xffffffffu, o1c[k][0], 1);
                     vol_vec<T>(o1c[k], ym, yp, o1m[k], o1p[k], unm[k], left, right, (uint32_t)km[k], l2, o2);
-                    if (x_ok && oy + r < g.ny) {
+                    if (r >= 0 && r < TY && x_ok && oy + r < g.ny) {
                         T *dst = out2 + (int64_t)(q - 1) * g.plane + (int64_t)(oy + r + 1) * g.pitch + g.xo + xv;
                         tb::st_v4_hint(dst, *(const uint4 *)o2, pol);
                     }
